@@ -1,0 +1,427 @@
+#!/usr/bin/env python
+"""ECL-CC on B200: Medges/s (device-timed) and % of HBM roofline, with the CPU oracle beside.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+
+One "step" = one full ECL-CC run (init_bin, hook_thread, hook_warp, hook_block, finalize)
+over the resident CSR of the workload (BASELINE.json configs; default C5 = Graph500
+Kronecker scale 27, edge factor 16, the config the metric's 1/2/4/8-GPU figure is quoted
+on).  For N > 1 (torchrun, one rank per GPU over NCCL) a step is the row-partitioned run
+(ecl_cc_run_rows) plus the binomial-tree forest merge, labels on rank 0 (strong scaling:
+the graph is fixed).  Prints ONE JSON line on rank 0.
+
+Metric: m / t, m = directed CSR entries (Table 2 "Edges*" convention).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+
+CONFIG_TEXT = {
+    "C1": "uniform random graph n=2^16, avg degree 4 (CSR, symmetric)",
+    "C2": "2D grid 4096x4096 with 10% random edge deletions",
+    "C3": "uniform random r4-2^23",
+    "C4": "R-MAT scale 24 edge factor 16",
+    "C5": "Kronecker/Graph500 scale 27 edge factor 16",
+}
+L2_BYTES = 126 * 2 ** 20
+METRIC = "Medges/s (device-timed) and % of HBM roofline at 1/2/4/8 B200 vs CPU oracle"
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.lines = []
+        if self.proc is not None:
+            time.sleep(0.1)
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [ln for ln in out.splitlines() if ln.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in getattr(self, "lines", []):
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for nm, val in zip(names, f[2:6]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": mx, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def build_graph(name: str, seed: int, device, scale_down: int = 0):
+    t0 = time.time()
+    g = gg.make_config(name, seed=seed, device=device, scale_down=scale_down)
+    torch.cuda.synchronize() if str(device).startswith("cuda") else None
+    return g, time.time() - t0
+
+
+def algorithmic_bytes(g, parent_init, hw):
+    """Per-phase algorithmic (compulsory, streamed) bytes of one run.
+    parent_init = Init3 parents (stop_after=1 run) on the device."""
+    n, m = g.n, g.m
+    s_idx = g.nindex.element_size()
+    deg = g.degrees()
+    v = torch.arange(n, device=g.nindex.device, dtype=torch.int64)
+    active = parent_init.to(torch.int64) != v
+    # Init3 reads row entries up to the first smaller one (rows are sorted by the
+    # generators, so that is 1 entry when one exists, else the whole row)
+    first = g.nlist[g.nindex[:-1].to(torch.int64).clamp(max=max(m - 1, 0))].to(torch.int64)
+    scanned = torch.where(deg == 0, torch.zeros_like(deg),
+                          torch.where(first < v, torch.ones_like(deg), deg))
+    t1, t2 = hw
+    thr = active & (deg <= t1)
+    fr = active & (deg > t1) & (deg <= t2)
+    bk = active & (deg > t2)
+    e_thr, e_fr, e_bk = (int(deg[x].sum()) for x in (thr, fr, bk))
+    n_fr, n_bk = int(fr.sum()), int(bk.sum())
+    b = {
+        "init_bin": s_idx * (n + 1) + 4 * n + 4 * int(scanned.sum()) + 8 * (n_fr + n_bk),
+        "hook_thread": s_idx * (n + 1) + 4 * n + 4 * e_thr,
+        "hook_warp": 8 * n_fr + 2 * s_idx * n_fr + 4 * e_fr,
+        "hook_block": 8 * n_bk + 2 * s_idx * n_bk + 4 * e_bk,
+        "finalize": 8 * n,
+    }
+    info = {"active": int(active.sum()), "thread_vertices": int(thr.sum()), "thread_entries": e_thr,
+            "warp_vertices": n_fr, "warp_entries": e_fr, "block_vertices": n_bk,
+            "block_entries": e_bk, "hooked_entries": None}
+    return b, info
+
+
+def flush_l2(buf):
+    buf.add_(1)
+
+
+def time_steps(fn, K, W, stream, flush_buf=None):
+    """W untimed warm-ups, then K steps each bracketed by CUDA events on `stream`."""
+    for _ in range(W):
+        fn()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(K)]
+    per = []
+    for i in range(K):
+        if flush_buf is not None:
+            with torch.cuda.stream(stream):
+                flush_l2(flush_buf)
+        evs[i][0].record(stream)
+        fn()
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    for a, b in evs:
+        per.append(a.elapsed_time(b))
+    return per
+
+
+def cpu_oracle_sample(config: str, seed: int, budget_s: float = 20.0):
+    """Time the oracle (O1 BFS, 1 thread) on a bounded sample of the same workload: the
+    same generator recipe scaled down until one run fits the budget."""
+    import oracle
+    sd = {"C1": 0, "C2": 0, "C3": 1, "C4": 3, "C5": 5}[config]
+    g, _ = build_graph(config, seed, "cuda" if torch.cuda.is_available() else "cpu", sd)
+    nidx, nl = g.numpy()
+    del g
+    oracle.build()
+    t0 = time.perf_counter()
+    _, ncc = oracle.bfs(nidx, nl)
+    dt = time.perf_counter() - t0
+    reps = 1
+    while dt * (reps + 1) / reps < budget_s and reps < 5 and dt < 2.0:
+        t1 = time.perf_counter()
+        oracle.bfs(nidx, nl)
+        dt += time.perf_counter() - t1
+        reps += 1
+    m = int(nl.shape[0])
+    return {"value": round(m * reps / dt / 1e6, 3), "unit": "Medges/s", "cores": 1,
+            "kind": "oracle",
+            "sample": f"{config} recipe at 1/2^{sd} scale (n={nidx.shape[0]-1}, m={m}), "
+                      f"O1 serial BFS, {reps} run(s), {dt:.2f} s, single thread of "
+                      f"{os.cpu_count()} host cores"}
+
+
+def run_reference(args):
+    """Reference arm = the CPU oracle as it stands, on a bounded sample of the workload."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    sd = {"C1": 0, "C2": 1, "C3": 2, "C4": 4, "C5": 6}[args.config]
+    g, _ = build_graph(args.config, args.seed, "cuda" if torch.cuda.is_available() else "cpu", sd)
+    nidx, nl = g.numpy()
+    del g
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle.bfs(nidx, nl)
+    per = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.bfs(nidx, nl)
+        per.append(time.perf_counter() - t0)
+    m = int(nl.shape[0])
+    tot = sum(per)
+    value = m * args.steps / tot / 1e6
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 3), "unit": "Medges/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * tot / args.steps, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": args.config, "description": CONFIG_TEXT[args.config],
+                   "sample_scale_down": sd, "n": int(nidx.shape[0] - 1), "m": m},
+        "cpu_baseline": {"value": round(value, 3), "unit": "Medges/s", "cores": 1,
+                         "kind": "oracle",
+                         "sample": f"{args.config} recipe at 1/2^{sd} scale, O1 serial BFS"},
+        "e2e": {"value": round(value, 3), "unit": "Medges/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C5", choices=sorted(CONFIG_TEXT))
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--load-mode", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--check", action="store_true", help="full oracle parity of the bench run")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    import paper_conf_hpdc_jaiganeshb18_b200 as ecl
+    if world > 1:
+        import torch.distributed as tdist
+        from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
+        tdist.init_process_group("nccl", device_id=dev)
+
+    g, gen_s = build_graph(args.config, args.seed, dev)
+    n, m = g.n, g.m
+    s_idx = g.nindex.element_size()
+    h = ecl.Handle(local)
+    h.set_option("load_mode", args.load_mode)
+    stream = torch.cuda.current_stream(dev)
+    labels = torch.empty(n, dtype=torch.int32, device=dev)
+    flush_buf = None if (m * 4 > 2 * L2_BYTES) else torch.zeros(64 * 2 ** 20, dtype=torch.int32,
+                                                                  device=dev)
+
+    # ---- algorithmic-bytes bookkeeping (outside the timed region) ----
+    h.set_option("stop_after", 1)
+    h.run(g.nindex, g.nlist, out=labels)
+    h.set_option("stop_after", 0)
+    alg, info = algorithmic_bytes(g, labels, (16, 352))
+    b_alg = s_idx * (n + 1) + 4 * m + 4 * n
+
+    if world == 1:
+        step = lambda: h.run(g.nindex, g.nlist, out=labels)  # noqa: E731
+    else:
+        bounds = edist.partition_rows(g.nindex, world)
+        lo, hi = bounds[rank], bounds[rank + 1]
+        idx_r, lst_r = edist.slice_rows(g.nindex, g.nlist, lo, hi)
+
+        def step():
+            parent = h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels)
+            edist.forest_merge(parent, h, chunks=4)
+
+    # ---- timed region ----
+    if world > 1:
+        tdist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        per = time_steps(step, args.steps, max(args.warmup, 3), stream, flush_buf)
+        if world > 1:
+            tdist.barrier()
+        torch.cuda.synchronize()
+    tot_ms = sum(per)
+    if world > 1:
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+    ms_step = tot_ms / args.steps
+    value = m / (ms_step * 1e-3) / 1e6
+
+    # ---- per-phase times (separate, event-instrumented runs; N=1 path) ----
+    phase = {}
+    if world == 1:
+        h.set_option("timing", 1)
+        acc = {k: 0.0 for k in ecl.PHASES}
+        reps = max(3, min(args.steps, 10))
+        for _ in range(reps):
+            if flush_buf is not None:
+                flush_l2(flush_buf)
+            h.run(g.nindex, g.nlist, out=labels)
+            for k, v in h.timing().items():
+                acc[k] += v
+        h.set_option("timing", 0)
+        phase = {k: v / reps for k, v in acc.items()}
+
+    # ---- parity of the bench output (invariants on the device; full oracle with --check) --
+    ok = None
+    if rank == 0:
+        lab = labels.to(torch.int64)
+        i1 = True
+        nidx64 = g.nindex.to(torch.int64)
+        chunk = 1 << 28
+        for a in range(0, m, chunk):
+            pos = torch.arange(a, min(m, a + chunk), device=dev, dtype=torch.int64)
+            rows = torch.searchsorted(nidx64, pos, right=True) - 1
+            i1 &= bool((lab[rows] == lab[g.nlist[a:a + chunk].to(torch.int64)]).all())
+            del pos, rows
+        del nidx64
+        ar = torch.arange(n, device=dev)
+        i2 = bool((lab <= ar).all()) and bool((lab[lab] == lab).all())
+        ok = {"I1": i1, "I2": i2, "components": int((lab == ar).sum())}
+        del lab, ar
+        if args.check:
+            import oracle
+            exp, ncc = oracle.bfs(*g.numpy())
+            ok["oracle_exact"] = bool(np.array_equal(labels.cpu().numpy(), exp))
+
+    # ---- end-to-end through the public API with host buffers ----
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hidx = g.nindex.cpu().pin_memory()
+        hlst = g.nlist.cpu().pin_memory()
+        hout = torch.empty(n, dtype=torch.int32).pin_memory()
+        h.run_host(hidx, hlst, out=hout)
+        ts = []
+        for _ in range(args.e2e_steps):
+            t0 = time.perf_counter()
+            h.run_host(hidx, hlst, out=hout)
+            ts.append(time.perf_counter() - t0)
+        e2e = {"value": round(m / (sum(ts) / len(ts)) / 1e6, 3), "unit": "Medges/s",
+               "h2d_bytes_per_step": int(hidx.numel() * hidx.element_size() + hlst.numel() * 4),
+               "d2h_bytes_per_step": int(n * 4), "steps": len(ts),
+               "ms_per_step": round(1e3 * sum(ts) / len(ts), 3)}
+        del hidx, hlst, hout
+
+    if rank != 0:
+        if world > 1:
+            tdist.barrier()
+            tdist.destroy_process_group()
+        return
+
+    peak, peak_src = peaks()
+    roof = None
+    if phase:
+        dom = max(phase, key=phase.get)
+        achieved = alg[dom] / (phase[dom] * 1e-3) / 1e9
+        roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1),
+                "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4),
+                "traffic": ncu_traffic(args.config, dom), "peak_source": peak_src,
+                "alg_bytes_per_launch": int(alg[dom]), "ms_per_launch": round(phase[dom], 4),
+                "path_alg_bytes": int(b_alg),
+                "path_frac": round(b_alg / (ms_step * 1e-3) / 1e9 / peak, 4)}
+    cpu = None
+    if world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_sample(args.config, args.seed)
+
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": "Medges/s", "n_gpus": world,
+        "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": round(ms_step, 4),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "int32", "data": "synthetic",
+        "config": {"workload": args.config, "description": CONFIG_TEXT[args.config],
+                   "seed": args.seed, "n": n, "m": m,
+                   "index_dtype": str(g.nindex.dtype).replace("torch.", ""),
+                   "l2": "inputs larger than L2" if flush_buf is None else
+                         "L2 flushed (256 MB write) between timed steps",
+                   "parallelism": f"rows{world}" if world > 1 else "single",
+                   "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info},
+        "gpu_launches": 5 * args.steps if world == 1 else None,
+        "clocks": clk.summary(),
+        "roofline": roof,
+        "phase_ms": {k: round(v, 4) for k, v in phase.items()},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "parity": ok,
+        "per_step_ms": [round(x, 4) for x in per],
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        tdist.barrier()
+        tdist.destroy_process_group()
+
+
+def ncu_traffic(config, kernel):
+    """DRAM bytes per launch of `kernel` from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(p))
+        return d[config][kernel]
+    except Exception:
+        return None
+
+
+if __name__ == "__main__":
+    main()

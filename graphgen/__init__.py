@@ -118,12 +118,14 @@ def csr_from_pairs(name: str, n: int, src: torch.Tensor, dst: torch.Tensor,
     """Symmetrize, drop self-loops, sort by (row, col), dedupe, build offsets.
 
     ``buckets`` > 1 splits the work by source-row range so that no single sort exceeds
-    ~1/buckets of the directed entries (needed for the 4e9-entry Kronecker config)."""
+    ~1/buckets of the directed entries (needed for the 4e9-entry Kronecker config); the
+    endpoint arrays stay in their input dtype and only one bucket's int64 keys exist at a
+    time."""
     device = src.device
-    src = src.to(torch.int64)
-    dst = dst.to(torch.int64)
-    keep = src != dst
-    src, dst = src[keep], dst[keep]
+    if src.dtype not in (torch.int32, torch.int64):
+        src = src.to(torch.int64)
+    if dst.dtype != src.dtype:
+        dst = dst.to(src.dtype)
     counts = torch.zeros(n, dtype=torch.int64, device=device)
     cols = []
     bounds = [(n * b) // buckets for b in range(buckets + 1)]
@@ -131,15 +133,21 @@ def csr_from_pairs(name: str, n: int, src: torch.Tensor, dst: torch.Tensor,
         lo, hi = bounds[b], bounds[b + 1]
         parts = []
         for a, c in ((src, dst), (dst, src)):
-            sel = (a >= lo) & (a < hi)
-            parts.append((a[sel] - lo) * n + c[sel])
+            sel = (a >= lo) & (a < hi) & (a != c)
+            aa = a[sel].to(torch.int64)
+            cc = c[sel].to(torch.int64)
+            del sel
+            parts.append((aa - lo) * n + cc)
+            del aa, cc
         keys = torch.unique(torch.cat(parts), sorted=True)
         del parts
         rows = keys // n
         counts[lo:hi] = torch.bincount(rows, minlength=hi - lo)
         cols.append((keys - rows * n).to(torch.int32))
         del keys, rows
-    nlist = torch.cat(cols) if cols else torch.zeros(0, dtype=torch.int32, device=device)
+    nlist = torch.cat(cols) if len(cols) > 1 else (
+        cols[0] if cols else torch.zeros(0, dtype=torch.int32, device=device))
+    del cols
     m = nlist.numel()
     if index_dtype is None:
         index_dtype = torch.int32 if m < 2 ** 31 else torch.int64

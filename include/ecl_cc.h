@@ -1,0 +1,164 @@
+/*
+ * ecl_cc.h — C ABI of the B200-native ECL-CC connected-components library (libecl_cc.so).
+ *
+ * The operation (PAPER.md = /root/reference/PAPER.md; "P:Lnnn" = its line nnn):
+ *   Given an undirected graph G = (V, E) in CSR form (§4: each undirected edge is
+ *   stored as two directed entries), "label each vertex with the ID of the component to
+ *   which it belongs" (§1).  The label written is the minimum vertex ID of the
+ *   component (the convention of P:L61 §1 / Fig. 1; reading R1) — the unique
+ *   fixed point the ECL-CC method (§3) reaches, so results are deterministic
+ *   and bit-exact across runs, launch configurations and GPU counts.
+ *
+ * Method (all on the GPU, hand-written CUDA for sm_100a):
+ *   init  : Init3 — parent[v] = first neighbour in adjacency order with a smaller ID,
+ *           else v (§3); vertices are binned by degree into a double-sided
+ *           worklist (§3: <=16 thread, 17..352 warp, >352 block).
+ *   hook  : asynchronous, lock-free union-find over every edge once, in one direction
+ *           (v > u), on representatives found with intermediate pointer jumping
+ *           (Fig. 5, Fig. 6).
+ *   final : single pointer jumping, parent[v] = root(v) (Fini3, §5.1).
+ *
+ * Conventions for every entry point:
+ *   - Vertex IDs are int32 in [0, n).  Offsets (nindex) are int32 (ecl_cc_run) or int64
+ *     (ecl_cc_run_i64); nindex has n+1 entries, nindex[0] == 0, nindex[n] == m, and is
+ *     non-decreasing.  nlist has m entries.
+ *   - Unless a name ends in _host, every pointer is a CUDA device pointer on the handle's
+ *     device.  The caller owns all of them; the library never frees them and keeps no
+ *     reference after the call returns.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Device
+ *     entry points only ENQUEUE work: no host synchronisation, no device->host copies.
+ *     Results are valid once the stream reaches that point.
+ *   - The graph must be symmetric (every (a,b) entry has a matching (b,a) entry); this is
+ *     a precondition, not checked by the run calls (R9).  ecl_cc_validate is the
+ *     opt-in checker.  Self-loops, duplicate entries and unsorted rows are accepted.
+ *   - Errors: argument errors return ECL_CC_ERR_INVALID_ARG before anything is enqueued;
+ *     CUDA launch/allocation errors return ECL_CC_ERR_CUDA / ECL_CC_ERR_OOM and the CUDA
+ *     error text is available from ecl_cc_last_error(h).  n == 0 is a no-op returning OK.
+ *   - A handle may be used by one host thread at a time.  It owns device scratch (the
+ *     double-sided worklist and counters, O(n)), allocated stream-ordered on first use,
+ *     grown on demand, and released by ecl_cc_destroy.
+ */
+#ifndef ECL_CC_H
+#define ECL_CC_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define ECL_CC_API __attribute__((visibility("default")))
+#else
+#define ECL_CC_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct ecl_cc_ctx *ecl_cc_handle;
+
+typedef enum {
+    ECL_CC_OK = 0,
+    ECL_CC_ERR_INVALID_ARG = 1,
+    ECL_CC_ERR_CUDA = 2,
+    ECL_CC_ERR_OOM = 3,
+    ECL_CC_ERR_INVALID_GRAPH = 4 /* only returned by ecl_cc_validate */
+} ecl_cc_status;
+
+/* Create a handle bound to CUDA device `device` (queries SM count / occupancy; no large
+ * allocations).  *out is set to NULL on failure. */
+ECL_CC_API ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device);
+
+/* Release the handle and its scratch.  NULL is a no-op.  Synchronises the handle's device
+ * before freeing. */
+ECL_CC_API ecl_cc_status ecl_cc_destroy(ecl_cc_handle h);
+
+/* Connected components of the whole graph (int32 offsets; requires m <= INT32_MAX).
+ *   n          number of vertices (>= 0)
+ *   m          number of directed CSR entries (== nindex[n])
+ *   nindex     n+1 offsets (device)
+ *   nlist      m neighbour IDs (device)
+ *   nstat_out  n labels out (device); also used as the union-find parent array during
+ *              the run, so it must not alias nindex/nlist.
+ * On completion nstat_out[v] = min{ w : w reachable from v }. */
+ECL_CC_API ecl_cc_status ecl_cc_run(ecl_cc_handle h, int32_t n, int64_t m, const int32_t *nindex,
+                         const int32_t *nlist, int32_t *nstat_out, void *stream);
+
+/* Same with int64 offsets (graphs with m > INT32_MAX, e.g. Graph500 scale 27). */
+ECL_CC_API ecl_cc_status ecl_cc_run_i64(ecl_cc_handle h, int32_t n, int64_t m, const int64_t *nindex,
+                             const int32_t *nlist, int32_t *nstat_out, void *stream);
+
+/* End-to-end convenience call on HOST buffers: copies nindex/nlist host->device into
+ * handle-owned device buffers, runs, copies the labels device->host, and synchronises
+ * `stream` before returning.  index_bytes is 4 (int32 offsets) or 8 (int64 offsets).
+ * Host buffers should be pinned (cudaHostAlloc / cudaHostRegister) for full PCIe speed. */
+ECL_CC_API ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex_host,
+                              int index_bytes, const int32_t *nlist_host,
+                              int32_t *labels_host, void *stream);
+
+/* ---- multi-GPU building blocks (the transport is the caller's NCCL process group) ----
+ * ecl_cc_run_rows: local forest of the rows [row_lo, row_hi) of a graph with n vertices.
+ *   nindex_rows  row_hi-row_lo+1 int64 offsets into nlist_rows, rebased so
+ *                nindex_rows[0] == 0 (device)
+ *   nlist_rows   the concatenated adjacency of those rows (device)
+ *   parent       n entries out (device): flattened min-ID labels of the subgraph formed by
+ *                the edges stored in these rows (every vertex outside them labels itself
+ *                unless joined through an edge).  Each undirected edge (a,b), a > b, is
+ *                hooked by the owner of row a only (Fig. 6 line 1 "if (v > u)").
+ * ecl_cc_merge: hook the edges (v, peer_labels[v - v_lo]) for v in [v_lo, v_hi) into the
+ *   forest `parent` (every v whose peer label differs from v; peer_labels is a flattened
+ *   min-ID labelling so peer_labels[v] <= v).  Does NOT flatten; call ecl_cc_finalize
+ *   once after the last merge chunk.
+ * ecl_cc_finalize: parent[v] = root(v) for all v (Fini3). */
+ECL_CC_API ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
+                              const int64_t *nindex_rows, const int32_t *nlist_rows,
+                              int32_t *parent, void *stream);
+ECL_CC_API ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_hi,
+                           const int32_t *peer_labels, int32_t *parent, void *stream);
+ECL_CC_API ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream);
+
+/* Debug checker (synchronises the stream): offsets monotone with nindex[0]==0 and
+ * nindex[n]==m, neighbour IDs in range, graph symmetric.  Returns ECL_CC_OK or
+ * ECL_CC_ERR_INVALID_GRAPH.  index_bytes is 4 or 8. */
+ECL_CC_API ecl_cc_status ecl_cc_validate(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex,
+                              int index_bytes, const int32_t *nlist, void *stream);
+
+/* ---- options (apply to later runs on this handle) ----------------------------------- */
+typedef enum {
+    ECL_CC_OPT_THRESH_THREAD = 1, /* max degree of the thread bin (paper: 16)           */
+    ECL_CC_OPT_THRESH_WARP = 2,   /* max degree of the warp bin (paper: 352)            */
+    ECL_CC_OPT_GRID_BLOCKS = 3,   /* override blocks per launch (0 = auto); race shaking */
+    ECL_CC_OPT_STOP_AFTER = 4,    /* debug: 1 = stop after init (nstat_out = Init3
+                                     parents), 2 = stop before finalize, 0 = full run    */
+    ECL_CC_OPT_LOAD_MODE = 5,     /* parent[] loads: 0 = ld.relaxed.gpu (L2-coherent),
+                                     1 = weak L1-cacheable loads (R7)          */
+    ECL_CC_OPT_TIMING = 6         /* 1 = record CUDA events between the phase kernels of
+                                     every run (read with ecl_cc_get_timing)             */
+} ecl_cc_option;
+ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
+
+/* Debug: copy the worklist of the most recent run (device->device, synchronises).
+ * front receives the warp-bin vertices, back the block-bin vertices (unordered sets);
+ * *nfront / *nback receive the counts.  Either buffer may be NULL to query counts only. */
+ECL_CC_API ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, int64_t *nfront,
+                                  int32_t *back, int64_t *nback);
+
+/* Debug counters, only non-zero in the ECL_CC_STATS build (libecl_cc_stats.so):
+ * [0] successful hook CASes, [1] failed hook CASes, [2] find_repres steps,
+ * [3] path-halving stores.  Synchronises; counters reset at the start of every run. */
+ECL_CC_API ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4]);
+
+/* Per-phase device time of the most recent full run with ECL_CC_OPT_TIMING set
+ * (synchronises on it): ms[0] init_bin (incl. the counter memset), ms[1] hook_thread,
+ * ms[2] hook_warp (worklist front), ms[3] hook_block (worklist back), ms[4] finalize. */
+ECL_CC_API ecl_cc_status ecl_cc_get_timing(ecl_cc_handle h, float ms[5]);
+
+/* 1 if this build counts statistics (ECL_CC_STATS), else 0. */
+ECL_CC_API int ecl_cc_stats_enabled(void);
+
+ECL_CC_API const char *ecl_cc_status_string(ecl_cc_status s);
+ECL_CC_API const char *ecl_cc_last_error(ecl_cc_handle h);
+ECL_CC_API const char *ecl_cc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ECL_CC_H */

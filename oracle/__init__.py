@@ -22,7 +22,24 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
-_LIB = os.path.join(_HERE, "liboracle.so")
+
+
+def _cpu_tag() -> str:
+    """-march=native code is host specific: key the library by the host CPU model."""
+    import hashlib
+    import platform
+    model = platform.machine()
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith(("model name", "flags")):
+                    model += line
+    except OSError:
+        pass
+    return hashlib.sha1(model.encode()).hexdigest()[:10]
+
+
+_LIB = os.path.join(_HERE, f"liboracle-{_cpu_tag()}.so")
 _lib = None
 
 

@@ -1,0 +1,291 @@
+"""B200-native ECL-CC connected components (Jaiganesh & Burtscher, HPDC '18).
+
+Thin Python binding over the C ABI of ``libecl_cc.so`` (declared in ``include/ecl_cc.h``).
+This module only marshals arguments: it checks dtypes/devices, passes raw pointers and the
+current CUDA stream, and raises on error.  Every step of the method runs in the library's
+CUDA kernels; there is no CPU or PyTorch fallback — if the library is missing, importing
+the binding works but every call raises ``RuntimeError`` (run ``__graft_entry__.build()``).
+
+Typical use::
+
+    import torch, paper_conf_hpdc_jaiganeshb18_b200 as ecl
+    labels = ecl.run(nindex, nlist)          # CUDA tensors; labels[v] = min ID of v's CC
+
+PAPER.md references: problem statement P:L45 (§1); method P:L135-L181 (§3).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+from typing import Optional
+
+import torch
+
+from . import build as _build
+
+__all__ = ["Handle", "run", "run_host", "EclCCError", "library_path", "OPT"]
+
+OPT = {
+    "thresh_thread": 1,
+    "thresh_warp": 2,
+    "grid_blocks": 3,
+    "stop_after": 4,
+    "load_mode": 5,
+    "timing": 6,
+}
+PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
+
+_STATUS = {0: "ok", 1: "invalid argument", 2: "CUDA error", 3: "out of device memory",
+           4: "invalid graph"}
+
+
+class EclCCError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"ecl_cc: {_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_libs = {}
+_lock = threading.Lock()
+
+
+def library_path(stats: bool = False) -> str:
+    return _build.lib_path("libecl_cc_stats.so" if stats else "libecl_cc.so")
+
+
+def _load(stats: bool = False) -> ctypes.CDLL:
+    with _lock:
+        if stats in _libs:
+            return _libs[stats]
+        path = library_path(stats)
+        if not os.path.exists(path):
+            raise RuntimeError(f"CUDA library {path} is not built; run "
+                               "`python -c 'import __graft_entry__ as g; g.build()'`")
+        lib = ctypes.CDLL(path)
+        P, I32, I64, INT = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int
+        sig = {
+            "ecl_cc_create": ([ctypes.POINTER(P), INT], INT),
+            "ecl_cc_destroy": ([P], INT),
+            "ecl_cc_run": ([P, I32, I64, P, P, P, P], INT),
+            "ecl_cc_run_i64": ([P, I32, I64, P, P, P, P], INT),
+            "ecl_cc_run_host": ([P, I32, I64, P, INT, P, P, P], INT),
+            "ecl_cc_run_rows": ([P, I32, I32, I32, P, P, P, P], INT),
+            "ecl_cc_merge": ([P, I32, I32, I32, P, P, P], INT),
+            "ecl_cc_finalize": ([P, I32, P, P], INT),
+            "ecl_cc_validate": ([P, I32, I64, P, INT, P, P], INT),
+            "ecl_cc_set_option": ([P, INT, I64], INT),
+            "ecl_cc_get_worklist": ([P, P, ctypes.POINTER(I64), P, ctypes.POINTER(I64)], INT),
+            "ecl_cc_get_stats": ([P, ctypes.POINTER(I64)], INT),
+            "ecl_cc_stats_enabled": ([], INT),
+            "ecl_cc_get_timing": ([P, ctypes.POINTER(ctypes.c_float)], INT),
+            "ecl_cc_status_string": ([INT], ctypes.c_char_p),
+            "ecl_cc_last_error": ([P], ctypes.c_char_p),
+            "ecl_cc_version": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(lib, name)
+            f.argtypes = args
+            f.restype = res
+        _libs[stats] = lib
+        return lib
+
+
+def _ptr(t: Optional[torch.Tensor]):
+    return ctypes.c_void_p(t.data_ptr()) if t is not None and t.numel() > 0 else ctypes.c_void_p(0)
+
+
+def _stream_ptr(stream, device) -> ctypes.c_void_p:
+    if stream is None:
+        stream = torch.cuda.current_stream(device)
+    if isinstance(stream, torch.cuda.Stream):
+        return ctypes.c_void_p(stream.cuda_stream)
+    return ctypes.c_void_p(int(stream))
+
+
+def _dev_tensor(t: torch.Tensor, name: str, dtypes, device: torch.device):
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name} must be a torch tensor")
+    if t.dtype not in dtypes:
+        raise TypeError(f"{name} must have dtype in {dtypes}, got {t.dtype}")
+    if t.device != device:
+        raise ValueError(f"{name} must live on {device}, got {t.device}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return t
+
+
+class Handle:
+    """Owns an ``ecl_cc_handle`` (device scratch + options) bound to one CUDA device."""
+
+    def __init__(self, device=None, stats: bool = False):
+        if not torch.cuda.is_available():
+            raise RuntimeError("ecl_cc needs a CUDA device (no CPU fallback exists)")
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None
+                                   else torch.device(device).index or 0)
+        self._lib = _load(stats)
+        h = ctypes.c_void_p()
+        st = self._lib.ecl_cc_create(ctypes.byref(h), self.device.index)
+        if st != 0:
+            raise EclCCError(st, "ecl_cc_create failed")
+        self._h = h
+
+    # -- plumbing ---------------------------------------------------------------------
+    def _check(self, st: int):
+        if st != 0:
+            raise EclCCError(st, self._lib.ecl_cc_last_error(self._h).decode())
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.ecl_cc_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    @property
+    def stats_enabled(self) -> bool:
+        return bool(self._lib.ecl_cc_stats_enabled())
+
+    def set_option(self, name: str, value: int) -> "Handle":
+        self._check(self._lib.ecl_cc_set_option(self._h, OPT[name], int(value)))
+        return self
+
+    # -- the operation ----------------------------------------------------------------
+    def run(self, nindex: torch.Tensor, nlist: torch.Tensor, out: Optional[torch.Tensor] = None,
+            stream=None) -> torch.Tensor:
+        """labels[v] = min vertex ID of v's component (enqueued on ``stream``)."""
+        d = self.device
+        _dev_tensor(nindex, "nindex", (torch.int32, torch.int64), d)
+        _dev_tensor(nlist, "nlist", (torch.int32,), d)
+        n = nindex.numel() - 1
+        if n < 0:
+            raise ValueError("nindex must hold n+1 offsets")
+        if out is None:
+            out = torch.empty(n, dtype=torch.int32, device=d)
+        _dev_tensor(out, "out", (torch.int32,), d)
+        if out.numel() != n:
+            raise ValueError("out must have n entries")
+        m = nlist.numel()
+        fn = self._lib.ecl_cc_run if nindex.dtype == torch.int32 else self._lib.ecl_cc_run_i64
+        self._check(fn(self._h, n, m, _ptr(nindex), _ptr(nlist), _ptr(out),
+                       _stream_ptr(stream, d)))
+        return out
+
+    def run_host(self, nindex, nlist, out=None, stream=None):
+        """End-to-end on host buffers (numpy arrays or CPU tensors, ideally pinned)."""
+        import numpy as np
+        idx = torch.as_tensor(nindex)
+        lst = torch.as_tensor(nlist)
+        if idx.device.type != "cpu" or lst.device.type != "cpu":
+            raise ValueError("run_host takes host buffers")
+        if idx.dtype not in (torch.int32, torch.int64) or lst.dtype != torch.int32:
+            raise TypeError("nindex must be int32/int64 and nlist int32")
+        idx, lst = idx.contiguous(), lst.contiguous()
+        n = idx.numel() - 1
+        if out is None:
+            out = torch.empty(n, dtype=torch.int32)
+        out = torch.as_tensor(out)
+        if out.dtype != torch.int32 or out.numel() != n or not out.is_contiguous():
+            raise ValueError("out must be a contiguous int32 host buffer with n entries")
+        self._check(self._lib.ecl_cc_run_host(
+            self._h, n, lst.numel(), _ptr(idx), 4 if idx.dtype == torch.int32 else 8,
+            _ptr(lst), _ptr(out), _stream_ptr(stream, self.device)))
+        return out
+
+    # -- multi-GPU building blocks ----------------------------------------------------
+    def run_rows(self, n: int, row_lo: int, row_hi: int, nindex_rows: torch.Tensor,
+                 nlist_rows: torch.Tensor, parent: Optional[torch.Tensor] = None, stream=None):
+        d = self.device
+        _dev_tensor(nindex_rows, "nindex_rows", (torch.int64,), d)
+        _dev_tensor(nlist_rows, "nlist_rows", (torch.int32,), d)
+        if nindex_rows.numel() != row_hi - row_lo + 1:
+            raise ValueError("nindex_rows must hold row_hi - row_lo + 1 offsets")
+        if parent is None:
+            parent = torch.empty(n, dtype=torch.int32, device=d)
+        _dev_tensor(parent, "parent", (torch.int32,), d)
+        self._check(self._lib.ecl_cc_run_rows(self._h, n, row_lo, row_hi, _ptr(nindex_rows),
+                                              _ptr(nlist_rows), _ptr(parent),
+                                              _stream_ptr(stream, d)))
+        return parent
+
+    def merge(self, parent: torch.Tensor, peer: torch.Tensor, v_lo: int = 0, stream=None):
+        d = self.device
+        _dev_tensor(parent, "parent", (torch.int32,), d)
+        _dev_tensor(peer, "peer", (torch.int32,), d)
+        n = parent.numel()
+        self._check(self._lib.ecl_cc_merge(self._h, n, v_lo, v_lo + peer.numel(), _ptr(peer),
+                                           _ptr(parent), _stream_ptr(stream, d)))
+        return parent
+
+    def finalize(self, parent: torch.Tensor, stream=None):
+        d = self.device
+        _dev_tensor(parent, "parent", (torch.int32,), d)
+        self._check(self._lib.ecl_cc_finalize(self._h, parent.numel(), _ptr(parent),
+                                              _stream_ptr(stream, d)))
+        return parent
+
+    # -- debug ------------------------------------------------------------------------
+    def validate(self, nindex: torch.Tensor, nlist: torch.Tensor, stream=None) -> bool:
+        d = self.device
+        _dev_tensor(nindex, "nindex", (torch.int32, torch.int64), d)
+        _dev_tensor(nlist, "nlist", (torch.int32,), d)
+        st = self._lib.ecl_cc_validate(self._h, nindex.numel() - 1, nlist.numel(), _ptr(nindex),
+                                       nindex.element_size(), _ptr(nlist),
+                                       _stream_ptr(stream, d))
+        if st == 4:
+            return False
+        self._check(st)
+        return True
+
+    def worklist(self):
+        nf, nb = ctypes.c_int64(0), ctypes.c_int64(0)
+        self._check(self._lib.ecl_cc_get_worklist(self._h, None, ctypes.byref(nf), None,
+                                                  ctypes.byref(nb)))
+        front = torch.empty(nf.value, dtype=torch.int32, device=self.device)
+        back = torch.empty(nb.value, dtype=torch.int32, device=self.device)
+        self._check(self._lib.ecl_cc_get_worklist(self._h, _ptr(front), ctypes.byref(nf),
+                                                  _ptr(back), ctypes.byref(nb)))
+        return front, back
+
+    def timing(self) -> dict:
+        """Per-phase device milliseconds of the last run (needs set_option('timing', 1))."""
+        arr = (ctypes.c_float * 5)()
+        self._check(self._lib.ecl_cc_get_timing(self._h, arr))
+        return dict(zip(PHASES, list(arr)))
+
+    def stats(self) -> dict:
+        arr = (ctypes.c_int64 * 4)()
+        self._check(self._lib.ecl_cc_get_stats(self._h, arr))
+        return {"cas_success": arr[0], "cas_fail": arr[1], "finds": arr[2],
+                "halving_stores": arr[3]}
+
+
+_default = {}
+
+
+def _handle(device) -> Handle:
+    key = torch.device(device).index if device is not None else torch.cuda.current_device()
+    if key not in _default:
+        _default[key] = Handle(key)
+    return _default[key]
+
+
+def run(nindex: torch.Tensor, nlist: torch.Tensor, out: Optional[torch.Tensor] = None,
+        stream=None) -> torch.Tensor:
+    """Connected-component labels (min vertex ID per component) of a CSR graph on CUDA."""
+    return _handle(nindex.device).run(nindex, nlist, out=out, stream=stream)
+
+
+def run_host(nindex, nlist, out=None, device=None):
+    """End-to-end on host arrays: H2D copy, run, D2H copy (synchronous)."""
+    return _handle(device).run_host(nindex, nlist, out=out)

@@ -1,0 +1,531 @@
+// ecl_cc.cu — host side of libecl_cc.so: the C ABI declared in include/ecl_cc.h.
+//
+// Launch sequence of one run (init, three compute kernels, finalize):
+//   memset(counters) -> init_bin -> hook_thread -> hook_range<front> -> hook_range<back>
+//   -> finalize, all enqueued on the caller's stream with no host synchronisation.
+#include "ecl_cc.h"
+#include "ecl_cc_kernels.cuh"
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <unordered_map>
+
+using namespace eclcc;
+
+struct ecl_cc_ctx {
+    int device = 0;
+    int sms = 0;
+    // scratch (device, grow-only)
+    int *wl = nullptr;
+    unsigned *ub = nullptr;
+    int cap = 0;
+    unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [2..5] stats
+    int *flags = nullptr;                 // validate flags
+    // end-to-end buffers (device, grow-only)
+    void *e2e_index = nullptr;
+    size_t e2e_index_bytes = 0;
+    int *e2e_list = nullptr;
+    size_t e2e_list_n = 0;
+    int *e2e_labels = nullptr;
+    size_t e2e_labels_n = 0;
+    // options
+    int t1 = 16, t2 = 352;
+    int grid_blocks = 0;
+    int stop_after = 0;
+    int load_mode = 0;
+    int timing = 0;                       // record per-kernel CUDA events
+    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    int ev_valid = 0;
+    // last run (for ecl_cc_get_worklist)
+    cudaStream_t last_stream = nullptr;
+    std::unordered_map<const void *, int> occ;
+    char err[512] = {0};
+};
+
+namespace {
+
+const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
+
+ecl_cc_status fail_cuda(ecl_cc_handle h, cudaError_t e, const char *where)
+{
+    if (h) snprintf(h->err, sizeof(h->err), "%s: %s (%s)", where, cudaGetErrorString(e),
+                    cudaGetErrorName(e));
+    return e == cudaErrorMemoryAllocation ? ECL_CC_ERR_OOM : ECL_CC_ERR_CUDA;
+}
+
+ecl_cc_status fail_arg(ecl_cc_handle h, const char *msg)
+{
+    if (h) snprintf(h->err, sizeof(h->err), "invalid argument: %s", msg);
+    return ECL_CC_ERR_INVALID_ARG;
+}
+
+#define CK(call, where)                                      \
+    do {                                                     \
+        cudaError_t e_ = (call);                             \
+        if (e_ != cudaSuccess) return fail_cuda(h, e_, where); \
+    } while (0)
+
+// Make `dev` current for the duration of a call, restoring the caller's device.
+struct DeviceGuard {
+    int prev = -1;
+    bool ok = true;
+    explicit DeviceGuard(int dev)
+    {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+    }
+    ~DeviceGuard()
+    {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+int blocks_per_sm(ecl_cc_handle h, const void *kernel)
+{
+    auto it = h->occ.find(kernel);
+    if (it != h->occ.end()) return it->second;
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kBlock, 0) != cudaSuccess || b < 1)
+        b = 1;
+    h->occ[kernel] = b;
+    return b;
+}
+
+// grid for a grid-stride kernel over `work` threads (or a persistent kernel if work < 0)
+int grid_for(ecl_cc_handle h, const void *kernel, long long work_threads)
+{
+    if (h->grid_blocks > 0) return h->grid_blocks;
+    const long long full = (long long)h->sms * blocks_per_sm(h, kernel);
+    if (work_threads < 0) return (int)full;
+    long long need = (work_threads + kBlock - 1) / kBlock;
+    if (need < 1) need = 1;
+    return (int)(need < full ? need : full);
+}
+
+ecl_cc_status ensure_scratch(ecl_cc_handle h, int need, cudaStream_t s)
+{
+    if (need <= h->cap) return ECL_CC_OK;
+    if (h->wl) CK(cudaFreeAsync(h->wl, s), "cudaFreeAsync(wl)");
+    if (h->ub) CK(cudaFreeAsync(h->ub, s), "cudaFreeAsync(ub)");
+    h->wl = nullptr;
+    h->ub = nullptr;
+    h->cap = 0;
+    CK(cudaMallocAsync((void **)&h->wl, sizeof(int) * (size_t)need, s), "cudaMallocAsync(wl)");
+    CK(cudaMallocAsync((void **)&h->ub, sizeof(unsigned) * (size_t)need, s), "cudaMallocAsync(ub)");
+    h->cap = need;
+    return ECL_CC_OK;
+}
+
+template <int MODE, typename idx_t>
+ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const idx_t *nindex,
+                          const int *nlist, int *parent, cudaStream_t s, bool rows_mode)
+{
+    ecl_cc_status st = ensure_scratch(h, nrows > 0 ? nrows : 1, s);
+    if (st != ECL_CC_OK) return st;
+    CK(cudaMemsetAsync(h->cnt, 0, 6 * sizeof(unsigned long long), s), "cudaMemsetAsync");
+    h->last_stream = s;
+
+    Params p;
+    p.n = n;
+    p.row_lo = row_lo;
+    p.nrows = nrows;
+    p.nindex = nindex;
+    p.nlist = nlist;
+    p.parent = parent;
+    p.wl = h->wl;
+    p.ub = h->ub;
+    p.cap = h->cap;
+    p.cnt = h->cnt;
+    p.stats = h->cnt + 2;
+    p.t1 = h->t1;
+    p.t2 = h->t2;
+
+    const bool tm = h->timing != 0;
+    if (tm) {
+        for (int i = 0; i < 6; i++)
+            if (!h->ev[i]) CK(cudaEventCreate(&h->ev[i]), "cudaEventCreate");
+        CK(cudaEventRecord(h->ev[0], s), "cudaEventRecord");
+    }
+    h->ev_valid = 0;
+    auto mark = [&](int i) {
+        if (tm) cudaEventRecord(h->ev[i], s);
+    };
+    if (rows_mode) {
+        auto k = identity_outside_kernel;
+        k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, row_lo, row_lo + nrows, parent);
+    }
+    {
+        auto k = init_bin_kernel<idx_t>;
+        k<<<grid_for(h, (const void *)k, nrows), kBlock, 0, s>>>(p);
+    }
+    mark(1);
+    if (h->stop_after != 1) {
+        {
+            auto k = hook_thread_kernel<MODE, idx_t>;
+            const long long tiles = (nrows + kWarp - 1) / kWarp;
+            k<<<grid_for(h, (const void *)k, tiles * kWarp), kBlock, 0, s>>>(p);
+        }
+        mark(2);
+        {
+            auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
+            k<<<grid_for(h, (const void *)k, -1), kBlock, 0, s>>>(p);
+        }
+        mark(3);
+        {
+            auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
+            k<<<grid_for(h, (const void *)k, -1), kBlock, 0, s>>>(p);
+        }
+        mark(4);
+        if (h->stop_after != 2) {
+            auto k = finalize_kernel<MODE>;
+            k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent);
+        }
+        mark(5);
+        if (tm && h->stop_after == 0) h->ev_valid = 1;
+    }
+    CK(cudaGetLastError(), "kernel launch");
+    return ECL_CC_OK;
+}
+
+template <typename idx_t>
+ecl_cc_status run_impl(ecl_cc_handle h, int32_t n, int64_t m, const idx_t *nindex,
+                       const int32_t *nlist, int32_t *out, void *stream, int row_lo,
+                       int nrows, bool rows_mode)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (n < 0) return fail_arg(h, "n < 0");
+    if (m < 0) return fail_arg(h, "m < 0");
+    if (n == 0) return ECL_CC_OK;
+    if (!out) return fail_arg(h, "null output/parent pointer");
+    if (nrows > 0 && !nindex) return fail_arg(h, "null nindex");
+    if (m > 0 && !nlist) return fail_arg(h, "null nlist");
+    if (m / kUnitFront + (long long)nrows >= (1LL << 32))
+        return fail_arg(h, "graph too large for 32-bit worklist unit counters");
+    DeviceGuard g(h->device);
+    if (!g.ok) return fail_arg(h, "cannot select the handle's device");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (h->load_mode == 1)
+        return launch_path<1, idx_t>(h, n, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    return launch_path<0, idx_t>(h, n, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+}
+
+}  // namespace
+
+extern "C" {
+
+ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device)
+{
+    if (!out) return ECL_CC_ERR_INVALID_ARG;
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
+        return ECL_CC_ERR_INVALID_ARG;
+    ecl_cc_handle h = new (std::nothrow) ecl_cc_ctx();
+    if (!h) return ECL_CC_ERR_OOM;
+    h->device = device;
+    DeviceGuard g(device);
+    cudaError_t e = cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
+    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, 8 * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc((void **)&h->flags, 4 * sizeof(int));
+    if (e != cudaSuccess) {
+        if (h->cnt) cudaFree(h->cnt);
+        delete h;
+        return e == cudaErrorMemoryAllocation ? ECL_CC_ERR_OOM : ECL_CC_ERR_CUDA;
+    }
+    *out = h;
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
+{
+    if (!h) return ECL_CC_OK;
+    {
+        DeviceGuard g(h->device);
+        cudaDeviceSynchronize();
+        if (h->wl) cudaFree(h->wl);
+        if (h->ub) cudaFree(h->ub);
+        if (h->cnt) cudaFree(h->cnt);
+        if (h->flags) cudaFree(h->flags);
+        if (h->e2e_index) cudaFree(h->e2e_index);
+        if (h->e2e_list) cudaFree(h->e2e_list);
+        if (h->e2e_labels) cudaFree(h->e2e_labels);
+        for (int i = 0; i < 6; i++)
+            if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+    }
+    delete h;
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_run(ecl_cc_handle h, int32_t n, int64_t m, const int32_t *nindex,
+                         const int32_t *nlist, int32_t *nstat_out, void *stream)
+{
+    if (m > INT32_MAX) return fail_arg(h, "m > INT32_MAX: use ecl_cc_run_i64");
+    return run_impl<int>(h, n, m, nindex, nlist, nstat_out, stream, 0, n, false);
+}
+
+ecl_cc_status ecl_cc_run_i64(ecl_cc_handle h, int32_t n, int64_t m, const int64_t *nindex,
+                             const int32_t *nlist, int32_t *nstat_out, void *stream)
+{
+    return run_impl<long long>(h, n, m, (const long long *)nindex, nlist, nstat_out, stream, 0,
+                               n, false);
+}
+
+ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
+                              const int64_t *nindex_rows, const int32_t *nlist_rows,
+                              int32_t *parent, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (row_lo < 0 || row_hi < row_lo || row_hi > n) return fail_arg(h, "bad row range");
+    // m of the slice is unknown on the host without a device read; callers pass the
+    // slice's adjacency, whose size only matters for the null-pointer check.
+    return run_impl<long long>(h, n, nlist_rows ? 1 : 0, (const long long *)nindex_rows,
+                               nlist_rows ? nlist_rows : (const int32_t *)nullptr, parent,
+                               stream, row_lo, row_hi - row_lo, true);
+}
+
+ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_hi,
+                           const int32_t *peer_labels, int32_t *parent, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (n < 0 || v_lo < 0 || v_hi < v_lo || v_hi > n) return fail_arg(h, "bad merge range");
+    if (v_hi == v_lo) return ECL_CC_OK;
+    if (!peer_labels || !parent) return fail_arg(h, "null pointer");
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    const int cnt = v_hi - v_lo;
+    if (h->load_mode == 1) {
+        auto k = merge_hook_kernel<1>;
+        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent
+#ifdef ECL_CC_STATS
+                                                                 , h->cnt + 2
+#endif
+        );
+    } else {
+        auto k = merge_hook_kernel<0>;
+        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent
+#ifdef ECL_CC_STATS
+                                                                 , h->cnt + 2
+#endif
+        );
+    }
+    CK(cudaGetLastError(), "merge_hook launch");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (n < 0) return fail_arg(h, "n < 0");
+    if (n == 0) return ECL_CC_OK;
+    if (!parent) return fail_arg(h, "null parent");
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    auto k = finalize_kernel<0>;
+    k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent);
+    CK(cudaGetLastError(), "finalize launch");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex_host,
+                              int index_bytes, const int32_t *nlist_host,
+                              int32_t *labels_host, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (index_bytes != 4 && index_bytes != 8) return fail_arg(h, "index_bytes must be 4 or 8");
+    if (n < 0 || m < 0) return fail_arg(h, "negative size");
+    if (n == 0) return ECL_CC_OK;
+    if (!nindex_host || !labels_host || (m > 0 && !nlist_host)) return fail_arg(h, "null pointer");
+    if (index_bytes == 4 && m > INT32_MAX) return fail_arg(h, "m > INT32_MAX with int32 offsets");
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t ib = (size_t)index_bytes * ((size_t)n + 1);
+    if (ib > h->e2e_index_bytes) {
+        if (h->e2e_index) CK(cudaFreeAsync(h->e2e_index, s), "cudaFreeAsync");
+        h->e2e_index = nullptr;
+        h->e2e_index_bytes = 0;
+        CK(cudaMallocAsync(&h->e2e_index, ib, s), "cudaMallocAsync(index)");
+        h->e2e_index_bytes = ib;
+    }
+    if ((size_t)m > h->e2e_list_n) {
+        if (h->e2e_list) CK(cudaFreeAsync(h->e2e_list, s), "cudaFreeAsync");
+        h->e2e_list = nullptr;
+        h->e2e_list_n = 0;
+        CK(cudaMallocAsync((void **)&h->e2e_list, sizeof(int) * (size_t)m, s), "cudaMallocAsync(list)");
+        h->e2e_list_n = (size_t)m;
+    }
+    if ((size_t)n > h->e2e_labels_n) {
+        if (h->e2e_labels) CK(cudaFreeAsync(h->e2e_labels, s), "cudaFreeAsync");
+        h->e2e_labels = nullptr;
+        h->e2e_labels_n = 0;
+        CK(cudaMallocAsync((void **)&h->e2e_labels, sizeof(int) * (size_t)n, s), "cudaMallocAsync(labels)");
+        h->e2e_labels_n = (size_t)n;
+    }
+    CK(cudaMemcpyAsync(h->e2e_index, nindex_host, ib, cudaMemcpyHostToDevice, s), "H2D nindex");
+    if (m > 0)
+        CK(cudaMemcpyAsync(h->e2e_list, nlist_host, sizeof(int) * (size_t)m, cudaMemcpyHostToDevice, s),
+           "H2D nlist");
+    ecl_cc_status st = index_bytes == 4
+        ? ecl_cc_run(h, n, m, (const int32_t *)h->e2e_index, h->e2e_list, h->e2e_labels, stream)
+        : ecl_cc_run_i64(h, n, m, (const int64_t *)h->e2e_index, h->e2e_list, h->e2e_labels, stream);
+    if (st != ECL_CC_OK) return st;
+    CK(cudaMemcpyAsync(labels_host, h->e2e_labels, sizeof(int) * (size_t)n, cudaMemcpyDeviceToHost, s),
+       "D2H labels");
+    CK(cudaStreamSynchronize(s), "cudaStreamSynchronize");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_validate(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex,
+                              int index_bytes, const int32_t *nlist, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (index_bytes != 4 && index_bytes != 8) return fail_arg(h, "index_bytes must be 4 or 8");
+    if (n < 0 || m < 0) return fail_arg(h, "negative size");
+    if (!nindex || (m > 0 && !nlist)) return fail_arg(h, "null pointer");
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    int flags = 0;
+    CK(cudaMemsetAsync(h->flags, 0, sizeof(int), s), "memset");
+    const int grid = (int)std::min<long long>(((long long)n + kBlock) / kBlock, 148LL * 8);
+    if (index_bytes == 4) {
+        validate_offsets_kernel<int><<<grid, kBlock, 0, s>>>(n, m, (const int *)nindex, h->flags);
+    } else {
+        validate_offsets_kernel<long long><<<grid, kBlock, 0, s>>>(n, m, (const long long *)nindex, h->flags);
+    }
+    CK(cudaMemcpyAsync(&flags, h->flags, sizeof(int), cudaMemcpyDeviceToHost, s), "D2H");
+    CK(cudaStreamSynchronize(s), "sync");
+    if (flags) {
+        snprintf(h->err, sizeof(h->err), "invalid graph: bad offsets");
+        return ECL_CC_ERR_INVALID_GRAPH;
+    }
+    if (n > 0) {
+        if (index_bytes == 4)
+            validate_rows_kernel<int><<<grid, kBlock, 0, s>>>(n, (const int *)nindex, nlist, h->flags);
+        else
+            validate_rows_kernel<long long><<<grid, kBlock, 0, s>>>(n, (const long long *)nindex, nlist, h->flags);
+        CK(cudaMemcpyAsync(&flags, h->flags, sizeof(int), cudaMemcpyDeviceToHost, s), "D2H");
+        CK(cudaStreamSynchronize(s), "sync");
+        if (flags & 2) {
+            snprintf(h->err, sizeof(h->err), "invalid graph: neighbour ID out of range");
+            return ECL_CC_ERR_INVALID_GRAPH;
+        }
+        const int sorted = (flags & 8) ? 0 : 1;
+        if (index_bytes == 4)
+            validate_symmetry_kernel<int><<<grid, kBlock, 0, s>>>(n, (const int *)nindex, nlist, sorted, h->flags);
+        else
+            validate_symmetry_kernel<long long><<<grid, kBlock, 0, s>>>(n, (const long long *)nindex, nlist, sorted, h->flags);
+        CK(cudaMemcpyAsync(&flags, h->flags, sizeof(int), cudaMemcpyDeviceToHost, s), "D2H");
+        CK(cudaStreamSynchronize(s), "sync");
+        if (flags & 4) {
+            snprintf(h->err, sizeof(h->err), "invalid graph: not symmetric");
+            return ECL_CC_ERR_INVALID_GRAPH;
+        }
+    }
+    CK(cudaGetLastError(), "validate launch");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    switch (option) {
+    case ECL_CC_OPT_THRESH_THREAD:
+        if (value < 0 || value > (1 << 30)) return fail_arg(h, "thread threshold");
+        h->t1 = (int)value;
+        break;
+    case ECL_CC_OPT_THRESH_WARP:
+        if (value < 0 || value > (1 << 30)) return fail_arg(h, "warp threshold");
+        h->t2 = (int)value;
+        break;
+    case ECL_CC_OPT_GRID_BLOCKS:
+        if (value < 0 || value > (1 << 24)) return fail_arg(h, "grid blocks");
+        h->grid_blocks = (int)value;
+        break;
+    case ECL_CC_OPT_STOP_AFTER:
+        if (value < 0 || value > 2) return fail_arg(h, "stop_after");
+        h->stop_after = (int)value;
+        break;
+    case ECL_CC_OPT_TIMING:
+        h->timing = value != 0;
+        break;
+    case ECL_CC_OPT_LOAD_MODE:
+        if (value < 0 || value > 1) return fail_arg(h, "load mode");
+        h->load_mode = (int)value;
+        break;
+    default:
+        return fail_arg(h, "unknown option");
+    }
+    if (h->t2 < h->t1) h->t2 = h->t1;
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, int64_t *nfront,
+                                  int32_t *back, int64_t *nback)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
+    cudaStream_t s = h->last_stream;
+    unsigned long long c[2] = {0, 0};
+    CK(cudaMemcpyAsync(c, h->cnt, sizeof(c), cudaMemcpyDeviceToHost, s), "D2H counters");
+    CK(cudaStreamSynchronize(s), "sync");
+    const long long nf = (long long)(unsigned)c[0], nb = (long long)(unsigned)c[1];
+    if (nfront) *nfront = nf;
+    if (nback) *nback = nb;
+    if (front && nf > 0)
+        CK(cudaMemcpyAsync(front, h->wl, sizeof(int) * nf, cudaMemcpyDeviceToDevice, s), "D2D front");
+    if (back && nb > 0)
+        CK(cudaMemcpyAsync(back, h->wl + h->cap - nb, sizeof(int) * nb, cudaMemcpyDeviceToDevice, s),
+           "D2D back");
+    CK(cudaStreamSynchronize(s), "sync");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4])
+{
+    if (!h || !out) return ECL_CC_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
+    unsigned long long c[4] = {0, 0, 0, 0};
+    CK(cudaStreamSynchronize(h->last_stream), "sync");
+    CK(cudaMemcpy(c, h->cnt + 2, sizeof(c), cudaMemcpyDeviceToHost), "D2H stats");
+    for (int i = 0; i < 4; i++) out[i] = (int64_t)c[i];
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_get_timing(ecl_cc_handle h, float ms[5])
+{
+    if (!h || !ms) return ECL_CC_ERR_INVALID_ARG;
+    if (!h->ev_valid) return fail_arg(h, "no timed full run recorded (set ECL_CC_OPT_TIMING)");
+    DeviceGuard g(h->device);
+    CK(cudaEventSynchronize(h->ev[5]), "cudaEventSynchronize");
+    for (int i = 0; i < 5; i++) CK(cudaEventElapsedTime(&ms[i], h->ev[i], h->ev[i + 1]), "elapsed");
+    return ECL_CC_OK;
+}
+
+int ecl_cc_stats_enabled(void)
+{
+#ifdef ECL_CC_STATS
+    return 1;
+#else
+    return 0;
+#endif
+}
+
+const char *ecl_cc_status_string(ecl_cc_status s)
+{
+    switch (s) {
+    case ECL_CC_OK: return "ok";
+    case ECL_CC_ERR_INVALID_ARG: return "invalid argument";
+    case ECL_CC_ERR_CUDA: return "CUDA error";
+    case ECL_CC_ERR_OOM: return "out of device memory";
+    case ECL_CC_ERR_INVALID_GRAPH: return "invalid graph";
+    }
+    return "unknown status";
+}
+
+const char *ecl_cc_last_error(ecl_cc_handle h) { return h ? h->err : "null handle"; }
+
+const char *ecl_cc_version(void) { return kVersion; }
+
+}  // extern "C"

@@ -1,0 +1,108 @@
+"""Multi-GPU ECL-CC: row-partitioned local forests merged over NCCL.
+
+Not in the paper (which is single-GPU); BASELINE.json's north_star adds it.  Each
+rank owns a contiguous row range of the CSR chosen so every rank holds ~m/G entries.  It
+builds a local forest of the edges stored in its rows with ``ecl_cc_run_rows`` (each
+undirected edge (a,b), a > b, is hooked only by the owner of row a: Fig. 6 line 1), then
+the forests are combined along a binomial tree: in round r the rank g with
+g mod 2^(r+1) == 2^r sends its flattened labels to g - 2^r, which receives them in chunks
+and hooks every (v, peer[v]) with ``ecl_cc_merge`` while the next chunk is in flight.
+Hook-once sufficiency makes the union of the forests' equivalence relations
+exact, so rank 0 ends with the same min-ID labels as a single-GPU run.
+
+The transport is a torch.distributed process group (NCCL on GPUs; gloo in the CPU tests);
+the compute is whatever ``ops`` object is passed (the CUDA ``Handle`` in the product).
+"""
+from __future__ import annotations
+
+from typing import List, Optional
+
+import torch
+import torch.distributed as dist
+
+
+def partition_rows(nindex: torch.Tensor, world: int) -> List[int]:
+    """Row bounds [b_0=0, ..., b_G=n] with ~m/G directed entries per range."""
+    nindex = nindex.to(torch.int64).cpu()
+    n = nindex.numel() - 1
+    m = int(nindex[-1])
+    targets = torch.tensor([(m * g) // world for g in range(1, world)], dtype=torch.int64)
+    cuts = torch.searchsorted(nindex, targets, right=False).clamp_(0, n).tolist()
+    bounds = [0] + cuts + [n]
+    for i in range(1, len(bounds)):
+        bounds[i] = max(bounds[i], bounds[i - 1])
+    return bounds
+
+
+def slice_rows(nindex: torch.Tensor, nlist: torch.Tensor, lo: int, hi: int):
+    """CSR slice of rows [lo, hi): int64 offsets rebased to 0, and the adjacency view."""
+    nindex = nindex.to(torch.int64)
+    a = int(nindex[lo])
+    b = int(nindex[hi])
+    return (nindex[lo:hi + 1] - a).contiguous(), nlist[a:b]
+
+
+def tree_schedule(world: int):
+    """Binomial-tree rounds: list of (round, sender, receiver)."""
+    out = []
+    step = 1
+    r = 0
+    while step < world:
+        for recv in range(0, world, 2 * step):
+            send = recv + step
+            if send < world:
+                out.append((r, send, recv))
+        step *= 2
+        r += 1
+    return out
+
+
+def forest_merge(parent: torch.Tensor, ops, group=None, chunks: int = 4,
+                 broadcast: bool = False) -> Optional[torch.Tensor]:
+    """Combine every rank's flattened forest ``parent`` (n labels) into rank 0's.
+
+    Returns the global labels on rank 0 (and on every rank if ``broadcast``), else None.
+    ``ops`` provides merge(parent, peer_chunk, v_lo) and finalize(parent)."""
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    n = parent.numel()
+    bounds = [(n * c) // chunks for c in range(chunks + 1)]
+    peer = None
+    for (_, send, recv) in tree_schedule(world):
+        if rank == send:
+            for c in range(chunks):
+                dist.send(parent[bounds[c]:bounds[c + 1]], dst=_g(group, recv), group=group)
+            break
+        if rank == recv:
+            if peer is None:
+                peer = torch.empty_like(parent)
+            works = [dist.irecv(peer[bounds[c]:bounds[c + 1]], src=_g(group, send), group=group)
+                     for c in range(chunks)]
+            for c in range(chunks):
+                works[c].wait()  # orders the compute stream after chunk c only
+                ops.merge(parent, peer[bounds[c]:bounds[c + 1]], bounds[c])
+            ops.finalize(parent)
+    if broadcast:
+        dist.broadcast(parent, src=_g(group, 0), group=group)
+        return parent
+    return parent if rank == 0 else None
+
+
+def _g(group, r):
+    return r if group is None else dist.get_global_rank(group, r)
+
+
+def run_distributed(nindex: torch.Tensor, nlist: torch.Tensor, handle, group=None,
+                    chunks: int = 4, broadcast: bool = False, bounds=None):
+    """Whole-graph CSR visible on every rank (device tensors); each rank processes its row
+    range, then the forests are merged.  Returns labels on rank 0 (all ranks if
+    ``broadcast``)."""
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    n = nindex.numel() - 1
+    if bounds is None:
+        bounds = partition_rows(nindex, world)
+    lo, hi = bounds[rank], bounds[rank + 1]
+    idx, lst = slice_rows(nindex, nlist, lo, hi)
+    parent = handle.run_rows(n, lo, hi, idx, lst)
+    return forest_merge(parent, handle, group=group, chunks=chunks, broadcast=broadcast)

@@ -1,0 +1,271 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact.
+
+The min-ID labelling is unique (R13), so every comparison is element-by-element
+equality with oracle O1 (BFS), plus the invariants I1-I3 on the GPU output.
+"""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+import graphgen as gg
+import oracle
+import paper_conf_hpdc_jaiganeshb18_b200 as ecl
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def h():
+    with ecl.Handle(0) as handle:
+        yield handle
+
+
+def gpu_labels(h, g, index_dtype=None, **opts):
+    g = g.to("cuda")
+    nindex = g.nindex if index_dtype is None else g.nindex.to(index_dtype)
+    for k, v in opts.items():
+        h.set_option(k, v)
+    try:
+        out = h.run(nindex, g.nlist)
+        torch.cuda.synchronize()
+    finally:
+        for k in opts:
+            h.set_option(k, {"thresh_thread": 16, "thresh_warp": 352}.get(k, 0))
+    return out.cpu().numpy()
+
+
+def assert_parity(h, g, **kw):
+    nidx, nl = g.numpy()
+    expect, ncc = oracle.bfs(nidx, nl)
+    got = gpu_labels(h, g, **kw)
+    if not np.array_equal(got, expect):
+        bad = np.nonzero(got != expect)[0]
+        raise AssertionError(f"{g.name}: {len(bad)} of {g.n} labels differ, first at v={bad[0]}: "
+                             f"gpu {got[bad[0]]} oracle {expect[bad[0]]}")
+    assert oracle.check(nidx, nl, got, ncc) == 0
+    return ncc
+
+
+# ---------------------------------------------------------------------------------------
+# hand-built graphs
+# ---------------------------------------------------------------------------------------
+def hand_graphs():
+    G = []
+    G.append(gg.from_edges(1, [], "single"))
+    G.append(gg.from_edges(7, [], "no_edges"))
+    G.append(gg.from_edges(5, [(4, 2), (2, 0), (0, 3), (3, 1)], "scrambled_path"))
+    ev = [(a, b) for a in range(0, 40, 2) for b in range(a + 2, 40, 2)]
+    od = [(a, b) for a in range(1, 40, 2) for b in range(a + 2, 40, 2)]
+    G.append(gg.from_edges(40, ev + od, "interleaved_cliques"))
+    G.append(gg.from_edges(10, [(3, 6), (7, 8), (6, 8)], "fig2"))
+    n = 5000
+    G.append(gg.from_edges(n, [(n - 1, i) for i in range(n - 1)], "star_center_last"))
+    G.append(gg.from_edges(n, [(0, i) for i in range(1, n)], "star_center_0"))
+    G.append(gg.from_edges(400, list(itertools.combinations(range(400), 2)), "K400"))
+    # rows of degree exactly 16 / 17 / 352 / 353 around the bin thresholds
+    edges = []
+    base = 0
+    for d in (15, 16, 17, 18, 351, 352, 353, 354):
+        hub = base + d  # hub has the largest ID so it is active and hooks all its leaves
+        edges += [(hub, base + i) for i in range(d)]
+        base += d + 1
+    G.append(gg.from_edges(base, edges, "degree_boundaries"))
+    # same, hubs with the smallest ID (inactive hubs: leaves hook into them)
+    edges = []
+    base = 0
+    for d in (16, 17, 352, 353):
+        edges += [(base, base + 1 + i) for i in range(d)]
+        base += d + 1
+    G.append(gg.from_edges(base, edges, "degree_boundaries_lowhub"))
+    return G
+
+
+@pytest.mark.parametrize("g", hand_graphs(), ids=lambda g: g.name)
+def test_hand_built(h, g):
+    assert_parity(h, g)
+
+
+def test_empty_graph(h):
+    out = h.run(torch.zeros(1, dtype=torch.int32, device="cuda"),
+                torch.zeros(0, dtype=torch.int32, device="cuda"))
+    assert out.numel() == 0
+
+
+def test_big_hub_chunked(h):
+    """One hub with 1.5M neighbours (spread over many warps), plus a second component."""
+    n = 1_500_002
+    src = torch.full((n - 2,), n - 2, dtype=torch.int64)
+    dst = torch.arange(n - 2, dtype=torch.int64)
+    g = gg.csr_from_pairs("hub1.5M", n, src, dst)
+    assert assert_parity(h, g) == 2
+
+
+def test_reversed_long_chain(h):
+    n = 1 << 20
+    v = torch.arange(1, n, dtype=torch.int64)
+    g = gg.csr_from_pairs("chain", n, v, v - 1)
+    assert assert_parity(h, g) == 1
+
+
+def test_fig3_pointer_jumping_shape(h):
+    """Long paths under Init3: a path whose IDs increase along it (each v's first smaller
+    neighbour is v-1), plus a path with IDs decreasing from the middle outwards."""
+    n = 100_000
+    a = list(range(0, n // 2 - 1))
+    e = [(i + 1, i) for i in a] + [(n // 2 + i, n // 2 + i + 1) for i in range(n // 2 - 1)]
+    e.append((n // 2, 0))
+    assert assert_parity(h, gg.from_edges(n, e, "two_paths")) == 1
+
+
+# ---------------------------------------------------------------------------------------
+# the five BASELINE configs, scaled so the oracle finishes in seconds
+# ---------------------------------------------------------------------------------------
+SMALL = {"C1": 0, "C2": 4, "C3": 4, "C4": 6, "C5": 10}
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("seed", [1, 2])
+def test_configs_scaled(h, name, seed):
+    g = gg.make_config(name, seed=seed, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g)
+
+
+@pytest.mark.parametrize("name", ["C1", "C3", "C4"])
+def test_row_shuffle_order_independence(h, name):
+    g = gg.make_config(name, seed=3, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, gg.shuffle_rows(g, seed=5))
+
+
+@pytest.mark.parametrize("grid", [1, 3, 148, 2000])
+@pytest.mark.parametrize("mode", [0, 1])
+def test_launch_config_sweep(h, grid, mode):
+    """Race shaking: very different interleavings must give the same labels."""
+    g = gg.make_config("C4", seed=4, scale_down=8, device="cuda")
+    assert_parity(h, g, grid_blocks=grid, load_mode=mode)
+
+
+@pytest.mark.parametrize("t1,t2", [(0, 0), (0, 10**9), (4, 8), (16, 352), (10**9, 10**9)])
+def test_threshold_sweep(h, t1, t2):
+    g = gg.make_config("C4", seed=5, scale_down=8, device="cuda")
+    assert_parity(h, g, thresh_thread=t1, thresh_warp=t2)
+
+
+@pytest.mark.parametrize("name", ["C2", "C4"])
+def test_int64_offsets(h, name):
+    g = gg.make_config(name, seed=1, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, index_dtype=torch.int64)
+
+
+# ---------------------------------------------------------------------------------------
+# intermediate, deterministic stages
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_init3_stage(h, name):
+    """stop_after=1 leaves Init3's parents in the output: exact per vertex."""
+    g = gg.make_config(name, seed=2, scale_down=SMALL[name], device="cuda")
+    g = gg.shuffle_rows(g, seed=9)
+    got = gpu_labels(h, g, stop_after=1)
+    assert np.array_equal(got, oracle.init3(*g.numpy()))
+
+
+def test_worklist_sets(h):
+    """Bins (reading R2/R3): front = active with 16 < deg <= 352, back = deg > 352."""
+    g = gg.make_config("C4", seed=1, scale_down=4, device="cuda")
+    gpu_labels(h, g)
+    front, back = h.worklist()
+    nidx, nl = g.numpy()
+    deg = np.diff(nidx.astype(np.int64))
+    active = oracle.init3(nidx, nl) != np.arange(g.n)
+    ef = np.nonzero(active & (deg > 16) & (deg <= 352))[0]
+    eb = np.nonzero(active & (deg > 352))[0]
+    assert np.array_equal(np.sort(front.cpu().numpy()), ef)
+    assert np.array_equal(np.sort(back.cpu().numpy()), eb)
+
+
+def test_run_host_end_to_end(h):
+    g = gg.make_config("C3", seed=1, scale_down=6)
+    nidx, nl = g.numpy()
+    out = h.run_host(torch.from_numpy(nidx).pin_memory(), torch.from_numpy(nl).pin_memory())
+    expect, _ = oracle.bfs(nidx, nl)
+    assert np.array_equal(out.numpy(), expect)
+
+
+def test_non_default_stream(h):
+    g = gg.make_config("C3", seed=2, scale_down=6, device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        out = h.run(g.nindex, g.nlist)
+    s.synchronize()
+    expect, _ = oracle.bfs(*g.numpy())
+    assert np.array_equal(out.cpu().numpy(), expect)
+
+
+def test_argument_errors(h):
+    idx = torch.zeros(5, dtype=torch.int32, device="cuda")
+    with pytest.raises(TypeError):
+        h.run(idx.float(), torch.zeros(0, dtype=torch.int32, device="cuda"))
+    lib = h._lib
+    assert lib.ecl_cc_run(h._h, -1, 0, None, None, None, None) == 1
+    assert lib.ecl_cc_run(h._h, 4, 2**31, idx.data_ptr(), None, None, None) == 1
+    assert lib.ecl_cc_run(h._h, 0, 0, None, None, None, None) == 0
+
+
+def test_validate(h):
+    g = gg.make_config("C1", seed=1, scale_down=4, device="cuda")
+    assert h.validate(g.nindex, g.nlist)
+    asym = gg.Graph("asym", 3, torch.tensor([0, 1, 1, 1], dtype=torch.int32, device="cuda"),
+                    torch.tensor([2], dtype=torch.int32, device="cuda"))
+    assert not h.validate(asym.nindex, asym.nlist)
+    bad = gg.Graph("oob", 2, torch.tensor([0, 1, 1], dtype=torch.int32, device="cuda"),
+                   torch.tensor([7], dtype=torch.int32, device="cuda"))
+    assert not h.validate(bad.nindex, bad.nlist)
+
+
+def test_stats_identity():
+    """-DECL_CC_STATS build: each successful hook CAS removes exactly one root, and
+    halving stores never create one, so #successful CAS == #Init3 roots - #CC (§8c)."""
+    with ecl.Handle(0, stats=True) as hs:
+        assert hs.stats_enabled
+        for name in ("C1", "C3", "C4"):
+            g = gg.make_config(name, seed=1, scale_down=SMALL[name], device="cuda")
+            got = gpu_labels(hs, g)
+            st = hs.stats()
+            nidx, nl = g.numpy()
+            expect, ncc = oracle.bfs(nidx, nl)
+            assert np.array_equal(got, expect)
+            roots = int((oracle.init3(nidx, nl) == np.arange(g.n)).sum())
+            assert st["cas_success"] == roots - ncc, (name, st, roots, ncc)
+
+
+def test_pre_finalize_forest_invariant(h):
+    """Before Fini3 every parent[x] <= x and the forest's roots are the component minima."""
+    g = gg.make_config("C3", seed=1, scale_down=6, device="cuda")
+    par = gpu_labels(h, g, stop_after=2)
+    assert np.all(par <= np.arange(g.n))
+    expect, ncc = oracle.bfs(*g.numpy())
+    assert int((par == np.arange(g.n)).sum()) == ncc
+
+
+# ---------------------------------------------------------------------------------------
+# multi-GPU math on one device: row partitions -> local forests -> sequential merges
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("G", [1, 2, 3, 4, 8])
+def test_fake_multi_gpu_merge(h, G):
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config("C4", seed=2, scale_down=7, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64.cpu(), G)
+    forests = []
+    for r in range(G):
+        lo, hi = bounds[r], bounds[r + 1]
+        idx, lst = dist.slice_rows(nindex64, g.nlist, lo, hi)
+        forests.append(h.run_rows(g.n, lo, hi, idx, lst))
+    acc = forests[0]
+    for f in forests[1:]:
+        h.merge(acc, f)
+    h.finalize(acc)
+    torch.cuda.synchronize()
+    assert np.array_equal(acc.cpu().numpy(), expect)
