@@ -247,7 +247,7 @@ def main():
     ap.add_argument("--config", default="C5", choices=sorted(CONFIG_TEXT))
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--load-mode", type=int, default=0)
+    ap.add_argument("--load-mode", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")

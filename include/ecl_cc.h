@@ -129,9 +129,11 @@ typedef enum {
     ECL_CC_OPT_STOP_AFTER = 4,    /* debug: 1 = stop after init (nstat_out = Init3
                                      parents), 2 = stop before finalize, 0 = full run    */
     ECL_CC_OPT_LOAD_MODE = 5,     /* parent[] loads: 0 = ld.relaxed.gpu (L2-coherent),
-                                     1 = weak L1-cacheable loads (R7)          */
-    ECL_CC_OPT_TIMING = 6         /* 1 = record CUDA events between the phase kernels of
+                                     1 (default) = weak L1-cacheable loads (R7)         */
+    ECL_CC_OPT_TIMING = 6,        /* 1 = record CUDA events between the phase kernels of
                                      every run (read with ecl_cc_get_timing)             */
+    ECL_CC_OPT_TTAS = 7           /* 1 (default) = load-test the target before every hook
+                                     CAS (test-and-test-and-set); 0 = bare CAS (Fig. 6)  */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

@@ -33,6 +33,7 @@ OPT = {
     "stop_after": 4,
     "load_mode": 5,
     "timing": 6,
+    "ttas": 7,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 
@@ -51,6 +52,8 @@ _lock = threading.Lock()
 
 
 def library_path(stats: bool = False) -> str:
+    if not stats and os.environ.get("ECL_CC_LIB"):   # dev A/B builds (tools/ab.sh)
+        return os.environ["ECL_CC_LIB"]
     return _build.lib_path("libecl_cc_stats.so" if stats else "libecl_cc.so")
 
 

@@ -34,7 +34,8 @@ struct ecl_cc_ctx {
     int t1 = 16, t2 = 352;
     int grid_blocks = 0;
     int stop_after = 0;
-    int load_mode = 0;
+    int load_mode = 1;
+    int ttas = 1;                         // test-and-test-and-set hooks
     int timing = 0;                       // record per-kernel CUDA events
     cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     int ev_valid = 0;
@@ -142,6 +143,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const i
     p.stats = h->cnt + 2;
     p.t1 = h->t1;
     p.t2 = h->t2;
+    p.ttas = h->ttas;
 
     const bool tm = h->timing != 0;
     if (tm) {
@@ -159,7 +161,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const i
     }
     {
         auto k = init_bin_kernel<idx_t>;
-        k<<<grid_for(h, (const void *)k, nrows), kBlock, 0, s>>>(p);
+        k<<<grid_for(h, (const void *)k, ((long long)nrows + kInitPerThread - 1) / kInitPerThread), kBlock, 0, s>>>(p);
     }
     mark(1);
     if (h->stop_after != 1) {
@@ -298,14 +300,14 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
     const int cnt = v_hi - v_lo;
     if (h->load_mode == 1) {
         auto k = merge_hook_kernel<1>;
-        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent
+        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
                                                                  , h->cnt + 2
 #endif
         );
     } else {
         auto k = merge_hook_kernel<0>;
-        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent
+        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
                                                                  , h->cnt + 2
 #endif
@@ -446,6 +448,9 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_STOP_AFTER:
         if (value < 0 || value > 2) return fail_arg(h, "stop_after");
         h->stop_after = (int)value;
+        break;
+    case ECL_CC_OPT_TTAS:
+        h->ttas = value != 0;
         break;
     case ECL_CC_OPT_TIMING:
         h->timing = value != 0;

@@ -1,0 +1,53 @@
+"""Dev tool: per-phase device times and debug counters for one config.
+
+    python tools/prof.py --config C3 [--mode 0|1] [--stats] [--reps 5] [--scale-down 0]
+"""
+import argparse
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+import paper_conf_hpdc_jaiganeshb18_b200 as ecl  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--mode", type=int, default=1)
+    ap.add_argument("--stats", action="store_true")
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--scale-down", type=int, default=0)
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--t1", type=int, default=16)
+    ap.add_argument("--t2", type=int, default=352)
+    ap.add_argument("--grid", type=int, default=0)
+    ap.add_argument("--ttas", type=int, default=1)
+    args = ap.parse_args()
+    g = gg.make_config(args.config, seed=args.seed, device="cuda", scale_down=args.scale_down)
+    h = ecl.Handle(0, stats=args.stats)
+    h.set_option("load_mode", args.mode).set_option("timing", 1)
+    h.set_option("thresh_thread", args.t1).set_option("thresh_warp", args.t2)
+    h.set_option("grid_blocks", args.grid).set_option("ttas", args.ttas)
+    out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    res = []
+    for _ in range(args.reps):
+        h.run(g.nindex, g.nlist, out=out)
+        t = h.timing()
+        t["total"] = sum(t.values())
+        res.append(t)
+    best = min(res, key=lambda r: r["total"])
+    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "n": g.n, "m": g.m, "mode": args.mode,
+            "best_ms": {k: round(v, 4) for k, v in best.items()},
+            "medges_s": round(g.m / best["total"] / 1e3, 1)}
+    if args.stats:
+        line["stats"] = h.stats()
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()
