@@ -96,6 +96,7 @@ ECL_CC_API ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, 
 
 /* ---- multi-GPU building blocks (the transport is the caller's NCCL process group) ----
  * ecl_cc_run_rows: local forest of the rows [row_lo, row_hi) of a graph with n vertices.
+ *   m_rows       entries of the slice (== nindex_rows[row_hi-row_lo])
  *   nindex_rows  row_hi-row_lo+1 int64 offsets into nlist_rows, rebased so
  *                nindex_rows[0] == 0 (device)
  *   nlist_rows   the concatenated adjacency of those rows (device)
@@ -109,8 +110,8 @@ ECL_CC_API ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, 
  *   once after the last merge chunk.
  * ecl_cc_finalize: parent[v] = root(v) for all v (Fini3). */
 ECL_CC_API ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
-                              const int64_t *nindex_rows, const int32_t *nlist_rows,
-                              int32_t *parent, void *stream);
+                              int64_t m_rows, const int64_t *nindex_rows,
+                              const int32_t *nlist_rows, int32_t *parent, void *stream);
 ECL_CC_API ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_hi,
                            const int32_t *peer_labels, int32_t *parent, void *stream);
 ECL_CC_API ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream);
@@ -128,12 +129,16 @@ typedef enum {
     ECL_CC_OPT_GRID_BLOCKS = 3,   /* override blocks per launch (0 = auto); race shaking */
     ECL_CC_OPT_STOP_AFTER = 4,    /* debug: 1 = stop after init (nstat_out = Init3
                                      parents), 2 = stop before finalize, 0 = full run    */
-    ECL_CC_OPT_LOAD_MODE = 5,     /* parent[] loads: 0 = ld.relaxed.gpu (L2-coherent),
-                                     1 (default) = weak L1-cacheable loads (R7)         */
+    ECL_CC_OPT_LOAD_MODE = 5,     /* parent[] loads: bit 0 set = weak L1-cacheable loads,
+                                     clear = ld.relaxed.gpu (R7); bit 1 = L2
+                                     policies (parent evict_last, adjacency evict_first) */
     ECL_CC_OPT_TIMING = 6,        /* 1 = record CUDA events between the phase kernels of
                                      every run (read with ecl_cc_get_timing)             */
-    ECL_CC_OPT_TTAS = 7           /* 1 (default) = load-test the target before every hook
+    ECL_CC_OPT_TTAS = 7,          /* 1 (default) = load-test the target before every hook
                                      CAS (test-and-test-and-set); 0 = bare CAS (Fig. 6)  */
+    ECL_CC_OPT_L2_FETCH = 8       /* cudaLimitMaxL2FetchGranularity hint in bytes (32, 64,
+                                     128) for the device; 0 = leave unchanged.  NOTE: a
+                                     device-wide setting that outlives the handle.       */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

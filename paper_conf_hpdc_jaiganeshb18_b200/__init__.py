@@ -34,6 +34,7 @@ OPT = {
     "load_mode": 5,
     "timing": 6,
     "ttas": 7,
+    "l2_fetch": 8,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 
@@ -73,7 +74,7 @@ def _load(stats: bool = False) -> ctypes.CDLL:
             "ecl_cc_run": ([P, I32, I64, P, P, P, P], INT),
             "ecl_cc_run_i64": ([P, I32, I64, P, P, P, P], INT),
             "ecl_cc_run_host": ([P, I32, I64, P, INT, P, P, P], INT),
-            "ecl_cc_run_rows": ([P, I32, I32, I32, P, P, P, P], INT),
+            "ecl_cc_run_rows": ([P, I32, I32, I32, I64, P, P, P, P], INT),
             "ecl_cc_merge": ([P, I32, I32, I32, P, P, P], INT),
             "ecl_cc_finalize": ([P, I32, P, P], INT),
             "ecl_cc_validate": ([P, I32, I64, P, INT, P, P], INT),
@@ -216,7 +217,8 @@ class Handle:
         if parent is None:
             parent = torch.empty(n, dtype=torch.int32, device=d)
         _dev_tensor(parent, "parent", (torch.int32,), d)
-        self._check(self._lib.ecl_cc_run_rows(self._h, n, row_lo, row_hi, _ptr(nindex_rows),
+        self._check(self._lib.ecl_cc_run_rows(self._h, n, row_lo, row_hi, nlist_rows.numel(),
+                                              _ptr(nindex_rows),
                                               _ptr(nlist_rows), _ptr(parent),
                                               _stream_ptr(stream, d)))
         return parent

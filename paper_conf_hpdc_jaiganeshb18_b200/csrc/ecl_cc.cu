@@ -84,22 +84,25 @@ struct DeviceGuard {
     }
 };
 
-int blocks_per_sm(ecl_cc_handle h, const void *kernel)
+int blocks_per_sm(ecl_cc_handle h, const void *kernel, size_t dsmem)
 {
     auto it = h->occ.find(kernel);
     if (it != h->occ.end()) return it->second;
+    if (dsmem > 0)
+        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
     int b = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kBlock, 0) != cudaSuccess || b < 1)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kBlock, dsmem) != cudaSuccess ||
+        b < 1)
         b = 1;
     h->occ[kernel] = b;
     return b;
 }
 
 // grid for a grid-stride kernel over `work` threads (or a persistent kernel if work < 0)
-int grid_for(ecl_cc_handle h, const void *kernel, long long work_threads)
+int grid_for(ecl_cc_handle h, const void *kernel, long long work_threads, size_t dsmem = 0)
 {
+    const long long full = (long long)h->sms * blocks_per_sm(h, kernel, dsmem);
     if (h->grid_blocks > 0) return h->grid_blocks;
-    const long long full = (long long)h->sms * blocks_per_sm(h, kernel);
     if (work_threads < 0) return (int)full;
     long long need = (work_threads + kBlock - 1) / kBlock;
     if (need < 1) need = 1;
@@ -121,8 +124,9 @@ ecl_cc_status ensure_scratch(ecl_cc_handle h, int need, cudaStream_t s)
 }
 
 template <int MODE, typename idx_t>
-ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const idx_t *nindex,
-                          const int *nlist, int *parent, cudaStream_t s, bool rows_mode)
+ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int nrows,
+                          const idx_t *nindex, const int *nlist, int *parent, cudaStream_t s,
+                          bool rows_mode)
 {
     ecl_cc_status st = ensure_scratch(h, nrows > 0 ? nrows : 1, s);
     if (st != ECL_CC_OK) return st;
@@ -133,6 +137,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const i
     p.n = n;
     p.row_lo = row_lo;
     p.nrows = nrows;
+    p.m = m;
     p.nindex = nindex;
     p.nlist = nlist;
     p.parent = parent;
@@ -168,17 +173,20 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, int row_lo, int nrows, const i
         {
             auto k = hook_thread_kernel<MODE, idx_t>;
             const long long tiles = (nrows + kWarp - 1) / kWarp;
-            k<<<grid_for(h, (const void *)k, tiles * kWarp), kBlock, 0, s>>>(p);
+            const size_t sm = hook_smem_bytes<idx_t>();
+            k<<<grid_for(h, (const void *)k, tiles * kWarp, sm), kBlock, sm, s>>>(p);
         }
         mark(2);
         {
             auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
-            k<<<grid_for(h, (const void *)k, -1), kBlock, 0, s>>>(p);
+            const size_t sm = hook_smem_bytes<idx_t>();
+            k<<<grid_for(h, (const void *)k, -1, sm), kBlock, sm, s>>>(p);
         }
         mark(3);
         {
             auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
-            k<<<grid_for(h, (const void *)k, -1), kBlock, 0, s>>>(p);
+            const size_t sm = hook_smem_bytes<idx_t>();
+            k<<<grid_for(h, (const void *)k, -1, sm), kBlock, sm, s>>>(p);
         }
         mark(4);
         if (h->stop_after != 2) {
@@ -209,9 +217,12 @@ ecl_cc_status run_impl(ecl_cc_handle h, int32_t n, int64_t m, const idx_t *ninde
     DeviceGuard g(h->device);
     if (!g.ok) return fail_arg(h, "cannot select the handle's device");
     cudaStream_t s = (cudaStream_t)stream;
-    if (h->load_mode == 1)
-        return launch_path<1, idx_t>(h, n, row_lo, nrows, nindex, nlist, out, s, rows_mode);
-    return launch_path<0, idx_t>(h, n, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    switch (h->load_mode) {
+    case 0: return launch_path<0, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    case 2: return launch_path<2, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    case 3: return launch_path<3, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    default: return launch_path<1, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    }
 }
 
 }  // namespace
@@ -276,15 +287,12 @@ ecl_cc_status ecl_cc_run_i64(ecl_cc_handle h, int32_t n, int64_t m, const int64_
 }
 
 ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
-                              const int64_t *nindex_rows, const int32_t *nlist_rows,
-                              int32_t *parent, void *stream)
+                              int64_t m_rows, const int64_t *nindex_rows,
+                              const int32_t *nlist_rows, int32_t *parent, void *stream)
 {
     if (!h) return ECL_CC_ERR_INVALID_ARG;
     if (row_lo < 0 || row_hi < row_lo || row_hi > n) return fail_arg(h, "bad row range");
-    // m of the slice is unknown on the host without a device read; callers pass the
-    // slice's adjacency, whose size only matters for the null-pointer check.
-    return run_impl<long long>(h, n, nlist_rows ? 1 : 0, (const long long *)nindex_rows,
-                               nlist_rows ? nlist_rows : (const int32_t *)nullptr, parent,
+    return run_impl<long long>(h, n, m_rows, (const long long *)nindex_rows, nlist_rows, parent,
                                stream, row_lo, row_hi - row_lo, true);
 }
 
@@ -449,6 +457,13 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         if (value < 0 || value > 2) return fail_arg(h, "stop_after");
         h->stop_after = (int)value;
         break;
+    case ECL_CC_OPT_L2_FETCH: {
+        if (value != 0 && value != 32 && value != 64 && value != 128)
+            return fail_arg(h, "L2 fetch granularity must be 0, 32, 64 or 128");
+        DeviceGuard g(h->device);
+        if (value) CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)value), "cudaDeviceSetLimit");
+        break;
+    }
     case ECL_CC_OPT_TTAS:
         h->ttas = value != 0;
         break;
@@ -456,7 +471,7 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         h->timing = value != 0;
         break;
     case ECL_CC_OPT_LOAD_MODE:
-        if (value < 0 || value > 1) return fail_arg(h, "load mode");
+        if (value < 0 || value > 3) return fail_arg(h, "load mode");
         h->load_mode = (int)value;
         break;
     default:
