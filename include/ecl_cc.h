@@ -136,9 +136,11 @@ typedef enum {
                                      every run (read with ecl_cc_get_timing)             */
     ECL_CC_OPT_TTAS = 7,          /* 1 (default) = load-test the target before every hook
                                      CAS (test-and-test-and-set); 0 = bare CAS (Fig. 6)  */
-    ECL_CC_OPT_L2_FETCH = 8       /* cudaLimitMaxL2FetchGranularity hint in bytes (32, 64,
+    ECL_CC_OPT_L2_FETCH = 8,      /* cudaLimitMaxL2FetchGranularity hint in bytes (32, 64,
                                      128) for the device; 0 = leave unchanged.  NOTE: a
                                      device-wide setting that outlives the handle.       */
+    ECL_CC_OPT_OCC_THREAD = 9,    /* blocks per SM of hook_thread (0 = max occupancy)     */
+    ECL_CC_OPT_OCC_RANGE = 10     /* blocks per SM of hook_warp / hook_block (0 = max)    */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

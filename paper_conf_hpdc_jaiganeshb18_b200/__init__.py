@@ -35,6 +35,8 @@ OPT = {
     "timing": 6,
     "ttas": 7,
     "l2_fetch": 8,
+    "occ_thread": 9,
+    "occ_range": 10,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

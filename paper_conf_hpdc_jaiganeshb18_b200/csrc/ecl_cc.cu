@@ -21,7 +21,8 @@ struct ecl_cc_ctx {
     int *wl = nullptr;
     unsigned *ub = nullptr;
     int cap = 0;
-    unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [2..5] stats
+    unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [2..5] stats,
+                                          // [8..9] int scheduling counters
     int *flags = nullptr;                 // validate flags
     // end-to-end buffers (device, grow-only)
     void *e2e_index = nullptr;
@@ -33,6 +34,7 @@ struct ecl_cc_ctx {
     // options
     int t1 = 16, t2 = 352;
     int grid_blocks = 0;
+    int occ_thread = 0, occ_range = 0;    // blocks per SM caps (0 = max occupancy)
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks
@@ -99,9 +101,12 @@ int blocks_per_sm(ecl_cc_handle h, const void *kernel, size_t dsmem)
 }
 
 // grid for a grid-stride kernel over `work` threads (or a persistent kernel if work < 0)
-int grid_for(ecl_cc_handle h, const void *kernel, long long work_threads, size_t dsmem = 0)
+int grid_for(ecl_cc_handle h, const void *kernel, long long work_threads, size_t dsmem = 0,
+             int occ_cap = 0)
 {
-    const long long full = (long long)h->sms * blocks_per_sm(h, kernel, dsmem);
+    int b = blocks_per_sm(h, kernel, dsmem);
+    if (occ_cap > 0 && occ_cap < b) b = occ_cap;
+    const long long full = (long long)h->sms * b;
     if (h->grid_blocks > 0) return h->grid_blocks;
     if (work_threads < 0) return (int)full;
     long long need = (work_threads + kBlock - 1) / kBlock;
@@ -130,7 +135,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
 {
     ecl_cc_status st = ensure_scratch(h, nrows > 0 ? nrows : 1, s);
     if (st != ECL_CC_OK) return st;
-    CK(cudaMemsetAsync(h->cnt, 0, 6 * sizeof(unsigned long long), s), "cudaMemsetAsync");
+    CK(cudaMemsetAsync(h->cnt, 0, 16 * sizeof(unsigned long long), s), "cudaMemsetAsync");
     h->last_stream = s;
 
     Params p;
@@ -146,6 +151,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.cap = h->cap;
     p.cnt = h->cnt;
     p.stats = h->cnt + 2;
+    p.sched = (int *)(h->cnt + 8);
     p.t1 = h->t1;
     p.t2 = h->t2;
     p.ttas = h->ttas;
@@ -174,19 +180,19 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             auto k = hook_thread_kernel<MODE, idx_t>;
             const long long tiles = (nrows + kWarp - 1) / kWarp;
             const size_t sm = hook_smem_bytes<idx_t>();
-            k<<<grid_for(h, (const void *)k, tiles * kWarp, sm), kBlock, sm, s>>>(p);
+            k<<<grid_for(h, (const void *)k, tiles * kWarp, sm, h->occ_thread), kBlock, sm, s>>>(p);
         }
         mark(2);
         {
             auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
             const size_t sm = hook_smem_bytes<idx_t>();
-            k<<<grid_for(h, (const void *)k, -1, sm), kBlock, sm, s>>>(p);
+            k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
         }
         mark(3);
         {
             auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
             const size_t sm = hook_smem_bytes<idx_t>();
-            k<<<grid_for(h, (const void *)k, -1, sm), kBlock, sm, s>>>(p);
+            k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
         }
         mark(4);
         if (h->stop_after != 2) {
@@ -241,7 +247,7 @@ ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device)
     h->device = device;
     DeviceGuard g(device);
     cudaError_t e = cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, 8 * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, 16 * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc((void **)&h->flags, 4 * sizeof(int));
     if (e != cudaSuccess) {
         if (h->cnt) cudaFree(h->cnt);
@@ -464,6 +470,14 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         if (value) CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)value), "cudaDeviceSetLimit");
         break;
     }
+    case ECL_CC_OPT_OCC_THREAD:
+        if (value < 0 || value > 64) return fail_arg(h, "occupancy cap");
+        h->occ_thread = (int)value;
+        break;
+    case ECL_CC_OPT_OCC_RANGE:
+        if (value < 0 || value > 64) return fail_arg(h, "occupancy cap");
+        h->occ_range = (int)value;
+        break;
     case ECL_CC_OPT_TTAS:
         h->ttas = value != 0;
         break;

@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--grid", type=int, default=0)
     ap.add_argument("--ttas", type=int, default=1)
     ap.add_argument("--l2fetch", type=int, default=0)
+    ap.add_argument("--occ-thread", type=int, default=0)
+    ap.add_argument("--occ-range", type=int, default=0)
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=args.seed, device="cuda", scale_down=args.scale_down)
     h = ecl.Handle(0, stats=args.stats)
@@ -35,6 +37,7 @@ def main():
     h.set_option("thresh_thread", args.t1).set_option("thresh_warp", args.t2)
     h.set_option("grid_blocks", args.grid).set_option("ttas", args.ttas)
     h.set_option("l2_fetch", args.l2fetch)
+    h.set_option("occ_thread", args.occ_thread).set_option("occ_range", args.occ_range)
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     res = []
     for _ in range(args.reps):
@@ -43,7 +46,7 @@ def main():
         t["total"] = sum(t.values())
         res.append(t)
     best = min(res, key=lambda r: r["total"])
-    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "l2fetch": args.l2fetch, "n": g.n, "m": g.m, "mode": args.mode,
+    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "n": g.n, "m": g.m, "mode": args.mode,
             "best_ms": {k: round(v, 4) for k, v in best.items()},
             "medges_s": round(g.m / best["total"] / 1e3, 1)}
     if args.stats:
