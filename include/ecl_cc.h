@@ -140,7 +140,15 @@ typedef enum {
                                      128) for the device; 0 = leave unchanged.  NOTE: a
                                      device-wide setting that outlives the handle.       */
     ECL_CC_OPT_OCC_THREAD = 9,    /* blocks per SM of hook_thread (0 = max occupancy)     */
-    ECL_CC_OPT_OCC_RANGE = 10     /* blocks per SM of hook_warp / hook_block (0 = max)    */
+    ECL_CC_OPT_OCC_RANGE = 10,    /* blocks per SM of hook_warp / hook_block (0 = max)    */
+    /* paper ablations; defaults are ECL-CC's */
+    ECL_CC_OPT_INIT = 11,         /* 3 = Init3 first smaller neighbour (default),
+                                     2 = Init2 smallest neighbour, 1 = Init1 own ID      */
+    ECL_CC_OPT_JUMP = 12,         /* 4 = intermediate (halving, default), 1 = multiple,
+                                     2 = single, 3 = none                                */
+    ECL_CC_OPT_FINI = 13,         /* 3 = single (default), 1 = intermediate, 2 = multiple */
+    ECL_CC_OPT_BATCH = 14         /* 1 (default) = batched two-hop gathers with early exit
+                                     at v_rep (R16/R19); 0 = one find per edge */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

@@ -37,6 +37,10 @@ OPT = {
     "l2_fetch": 8,
     "occ_thread": 9,
     "occ_range": 10,
+    "init": 11,
+    "jump": 12,
+    "fini": 13,
+    "batch": 14,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

@@ -35,6 +35,8 @@ struct ecl_cc_ctx {
     int t1 = 16, t2 = 352;
     int grid_blocks = 0;
     int occ_thread = 0, occ_range = 0;    // blocks per SM caps (0 = max occupancy)
+    int init_mode = 3, jump = 4, fini = 3; // paper ablation variants (defaults = ECL-CC)
+    int batch = 1;                        // batched two-hop gathers (R16, R19)
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks
@@ -155,6 +157,9 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.t1 = h->t1;
     p.t2 = h->t2;
     p.ttas = h->ttas;
+    p.init_mode = h->init_mode;
+    p.jump = h->jump;
+    p.batch = h->batch;
 
     const bool tm = h->timing != 0;
     if (tm) {
@@ -197,7 +202,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         mark(4);
         if (h->stop_after != 2) {
             auto k = finalize_kernel<MODE>;
-            k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent);
+            k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
         }
         mark(5);
         if (tm && h->stop_after == 0) h->ev_valid = 1;
@@ -340,7 +345,7 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
     auto k = finalize_kernel<0>;
-    k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent);
+    k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
     CK(cudaGetLastError(), "finalize launch");
     return ECL_CC_OK;
 }
@@ -477,6 +482,21 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_OCC_RANGE:
         if (value < 0 || value > 64) return fail_arg(h, "occupancy cap");
         h->occ_range = (int)value;
+        break;
+    case ECL_CC_OPT_INIT:
+        if (value < 1 || value > 3) return fail_arg(h, "init variant must be 1, 2 or 3");
+        h->init_mode = (int)value;
+        break;
+    case ECL_CC_OPT_JUMP:
+        if (value < 1 || value > 4) return fail_arg(h, "jump variant must be 1..4");
+        h->jump = (int)value;
+        break;
+    case ECL_CC_OPT_FINI:
+        if (value < 1 || value > 3) return fail_arg(h, "fini variant must be 1, 2 or 3");
+        h->fini = (int)value;
+        break;
+    case ECL_CC_OPT_BATCH:
+        h->batch = value != 0;
         break;
     case ECL_CC_OPT_TTAS:
         h->ttas = value != 0;

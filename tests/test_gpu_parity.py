@@ -15,6 +15,9 @@ import paper_conf_hpdc_jaiganeshb18_b200 as ecl
 
 pytestmark = pytest.mark.gpu
 
+DEFAULTS = {"thresh_thread": 16, "thresh_warp": 352, "load_mode": 1, "ttas": 1, "init": 3,
+            "jump": 4, "fini": 3}
+
 
 @pytest.fixture(scope="module")
 def h():
@@ -32,7 +35,7 @@ def gpu_labels(h, g, index_dtype=None, **opts):
         torch.cuda.synchronize()
     finally:
         for k in opts:
-            h.set_option(k, {"thresh_thread": 16, "thresh_warp": 352}.get(k, 0))
+            h.set_option(k, DEFAULTS.get(k, 0))
     return out.cpu().numpy()
 
 
@@ -269,3 +272,32 @@ def test_fake_multi_gpu_merge(h, G):
     h.finalize(acc)
     torch.cuda.synchronize()
     assert np.array_equal(acc.cpu().numpy(), expect)
+
+
+# ---------------------------------------------------------------------------------------
+# paper ablations: every Init/Jump/Fini variant must give the same labels
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("init", [1, 2, 3])
+@pytest.mark.parametrize("jump", [1, 2, 3, 4])
+@pytest.mark.parametrize("fini", [1, 2, 3])
+@pytest.mark.parametrize("name", ["C2", "C4"])
+def test_ablation_variants(h, name, init, jump, fini):
+    g = gg.make_config(name, seed=6, scale_down={"C2": 6, "C4": 8}[name], device="cuda")
+    g = gg.shuffle_rows(g, seed=2)
+    assert_parity(h, g, init=init, jump=jump, fini=fini)
+
+
+@pytest.mark.parametrize("init", [1, 2])
+def test_init_variant_stage(h, init):
+    """Init1 leaves parent[v] = v; Init2 the smallest neighbour if smaller."""
+    g = gg.shuffle_rows(gg.make_config("C4", seed=3, scale_down=8, device="cuda"), seed=4)
+    got = gpu_labels(h, g, stop_after=1, init=init)
+    nidx, nl = g.numpy()
+    if init == 1:
+        assert np.array_equal(got, np.arange(g.n))
+    else:
+        deg = np.diff(nidx.astype(np.int64))
+        rows = np.repeat(np.arange(g.n), deg)
+        mn = np.arange(g.n)
+        np.minimum.at(mn, rows, nl)
+        assert np.array_equal(got, mn)
