@@ -176,11 +176,11 @@ def time_steps(fn, K, W, stream, flush_buf=None):
     return per
 
 
-def cpu_oracle_sample(config: str, seed: int, budget_s: float = 12.0):
+def cpu_oracle_sample(config: str, seed: int, budget_s: float = 15.0):
     """Time the oracle (O1 BFS, 1 thread) on a bounded sample of the same workload: the
     same generator recipe scaled down until one run fits the budget."""
     import oracle
-    sd = {"C1": 0, "C2": 0, "C3": 0, "C4": 2, "C5": 4}[config]
+    sd = {"C1": 0, "C2": 0, "C3": 0, "C4": 1, "C5": 3}[config]
     g, _ = build_graph(config, seed, "cuda" if torch.cuda.is_available() else "cpu", sd)
     nidx, nl = g.numpy()
     del g

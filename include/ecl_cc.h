@@ -147,8 +147,10 @@ typedef enum {
     ECL_CC_OPT_JUMP = 12,         /* 4 = intermediate (halving, default), 1 = multiple,
                                      2 = single, 3 = none                                */
     ECL_CC_OPT_FINI = 13,         /* 3 = single (default), 1 = intermediate, 2 = multiple */
-    ECL_CC_OPT_BATCH = 14         /* 1 (default) = batched two-hop gathers with early exit
+    ECL_CC_OPT_BATCH = 14,        /* 1 (default) = batched two-hop gathers with early exit
                                      at v_rep (R16/R19); 0 = one find per edge */
+    ECL_CC_OPT_FILTER = 15        /* anchor-tree membership bitmap (R21): 0 off,
+                                     1 on, 2 (default) = on when 4n > 128 MB             */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

@@ -41,6 +41,7 @@ OPT = {
     "jump": 12,
     "fini": 13,
     "batch": 14,
+    "filter": 15,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

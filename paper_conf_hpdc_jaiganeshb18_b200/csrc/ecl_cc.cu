@@ -37,6 +37,9 @@ struct ecl_cc_ctx {
     int occ_thread = 0, occ_range = 0;    // blocks per SM caps (0 = max occupancy)
     int init_mode = 3, jump = 4, fini = 3; // paper ablation variants (defaults = ECL-CC)
     int batch = 1;                        // batched two-hop gathers (R16, R19)
+    int filter = 2;                       // R21 membership filter: 0 off, 1 on, 2 auto
+    unsigned *gbits = nullptr;            // R21 bitmap (grow-only)
+    size_t gbits_words = 0;
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks
@@ -160,6 +163,24 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.init_mode = h->init_mode;
     p.jump = h->jump;
     p.batch = h->batch;
+    p.anchor = h->cnt + 10;
+    p.gbits = nullptr;
+    {
+        // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
+        const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
+        if (on) {
+            const size_t words = ((size_t)n + 31) / 32;
+            if (words > h->gbits_words) {
+                if (h->gbits) CK(cudaFreeAsync(h->gbits, s), "cudaFreeAsync(gbits)");
+                h->gbits = nullptr;
+                h->gbits_words = 0;
+                CK(cudaMallocAsync((void **)&h->gbits, words * 4, s), "cudaMallocAsync(gbits)");
+                h->gbits_words = words;
+            }
+            CK(cudaMemsetAsync(h->gbits, 0, words * 4, s), "cudaMemsetAsync(gbits)");
+            p.gbits = h->gbits;
+        }
+    }
 
     const bool tm = h->timing != 0;
     if (tm) {
@@ -276,6 +297,7 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
         if (h->e2e_index) cudaFree(h->e2e_index);
         if (h->e2e_list) cudaFree(h->e2e_list);
         if (h->e2e_labels) cudaFree(h->e2e_labels);
+        if (h->gbits) cudaFree(h->gbits);
         for (int i = 0; i < 6; i++)
             if (h->ev[i]) cudaEventDestroy(h->ev[i]);
     }
@@ -494,6 +516,10 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_FINI:
         if (value < 1 || value > 3) return fail_arg(h, "fini variant must be 1, 2 or 3");
         h->fini = (int)value;
+        break;
+    case ECL_CC_OPT_FILTER:
+        if (value < 0 || value > 2) return fail_arg(h, "filter must be 0, 1 or 2");
+        h->filter = (int)value;
         break;
     case ECL_CC_OPT_BATCH:
         h->batch = value != 0;

@@ -16,7 +16,7 @@ import paper_conf_hpdc_jaiganeshb18_b200 as ecl
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"thresh_thread": 16, "thresh_warp": 352, "load_mode": 1, "ttas": 1, "init": 3,
-            "jump": 4, "fini": 3}
+            "jump": 4, "fini": 3, "batch": 1, "filter": 2}
 
 
 @pytest.fixture(scope="module")
@@ -301,3 +301,19 @@ def test_init_variant_stage(h, init):
         mn = np.arange(g.n)
         np.minimum.at(mn, rows, nl)
         assert np.array_equal(got, mn)
+
+
+# ---------------------------------------------------------------------------------------
+# R21 anchor-tree membership filter (forced on at small sizes; auto-on only for 4n > 128 MB)
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("grid", [0, 3, 148])
+def test_membership_filter(h, name, grid):
+    g = gg.make_config(name, seed=8, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, filter=1, grid_blocks=grid)
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2, 3])
+def test_load_modes_with_filter(h, mode):
+    g = gg.make_config("C5", seed=9, scale_down=9, device="cuda")
+    assert_parity(h, g, filter=1, load_mode=mode)

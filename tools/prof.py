@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--l2fetch", type=int, default=0)
     ap.add_argument("--occ-thread", type=int, default=0)
     ap.add_argument("--batch", type=int, default=1)
+    ap.add_argument("--filter", type=int, default=2)
     ap.add_argument("--jump", type=int, default=4)
     ap.add_argument("--init", type=int, default=3)
     ap.add_argument("--fini", type=int, default=3)
@@ -43,6 +44,7 @@ def main():
     h.set_option("l2_fetch", args.l2fetch)
     h.set_option("occ_thread", args.occ_thread).set_option("occ_range", args.occ_range)
     h.set_option("batch", args.batch).set_option("jump", args.jump)
+    h.set_option("filter", args.filter)
     h.set_option("init", args.init).set_option("fini", args.fini)
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     res = []
@@ -52,7 +54,7 @@ def main():
         t["total"] = sum(t.values())
         res.append(t)
     best = min(res, key=lambda r: r["total"])
-    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "n": g.n, "m": g.m, "mode": args.mode,
+    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "n": g.n, "m": g.m, "mode": args.mode,
             "best_ms": {k: round(v, 4) for k, v in best.items()},
             "medges_s": round(g.m / best["total"] / 1e3, 1)}
     if args.stats:
