@@ -94,6 +94,62 @@ ECL_CC_API ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, 
                               int index_bytes, const int32_t *nlist_host,
                               int32_t *labels_host, void *stream);
 
+/* Connected components plus a spanning forest (the union-find use the
+ * paper names next).  Labels are written to labels_out exactly as ecl_cc_run
+ * does.  For every vertex x that is not its component's minimum, (tree_a[x], tree_b[x])
+ * is a CSR edge, and these n - #components edges form a spanning forest of the graph
+ * (one spanning tree per component); for component minima both entries are -1.
+ * The edges are the Init edges (x, parent[x]) of the initialisation plus, for
+ * every successful hook CAS of Fig. 6 (lines 9/14) that made a root x a child, the edge
+ * being hooked — it joins exactly the two trees the CAS merges.  The forest is one
+ * valid answer of many (it depends on the race order); the labels are unique.
+ *   index_bytes  4 (nindex is int32, m <= INT32_MAX) or 8 (int64)
+ *   tree_a/b     n int32 each (device), caller-owned.
+ * Same errors and asynchrony as ecl_cc_run. */
+ECL_CC_API ecl_cc_status ecl_cc_spanning_forest(ecl_cc_handle h, int32_t n, int64_t m,
+                                                const void *nindex, int index_bytes,
+                                                const int32_t *nlist, int32_t *labels_out,
+                                                int32_t *tree_a, int32_t *tree_b, void *stream);
+
+/* ---- input preparation beside the hot path ----------------------------
+ * ecl_cc_build_csr: the symmetric CSR ECL-CC consumes, built on the GPU from an undirected
+ * edge list the way the paper prepared its inputs (§4): self-loops are removed,
+ * multiple edges between the same two vertices are merged, missing back edges are added,
+ * and each undirected edge becomes two directed entries.  Rows come out ascending.
+ *   n              number of vertices; every src/dst ID must be in [0, n)
+ *   num_edges      pairs in src/dst (device, int32 each); (a,b) and (b,a) are the same edge
+ *   nindex_out     n+1 int64 offsets (device, caller-owned)
+ *   nlist_out      int32 entries (device, caller-owned), room for nlist_capacity entries;
+ *                  2*num_edges always suffices
+ *   m_out          HOST int64: entries written (== nindex_out[n])
+ * Synchronises `stream` (the entry count is returned to the host).  Scratch (2 x 16 bytes
+ * per pair + CUB temp) is owned by the handle, grow-only.  Errors: INVALID_GRAPH if an ID
+ * is out of range; INVALID_ARG (with *m_out = the needed count) if nlist_capacity is too
+ * small.  The sort and duplicate removal use CUB (cub::DeviceRadixSort, DeviceSelect). */
+ECL_CC_API ecl_cc_status ecl_cc_build_csr(ecl_cc_handle h, int32_t n, int64_t num_edges,
+                                          const int32_t *src, const int32_t *dst,
+                                          int64_t *nindex_out, int32_t *nlist_out,
+                                          int64_t nlist_capacity, int64_t *m_out, void *stream);
+
+/* Host readers (no handle, no GPU): an undirected edge list in malloc'ed host arrays
+ * (*src_out, *dst_out; release each with ecl_cc_free_host).  Edges are returned as stored
+ * (loops / duplicates / one direction only); pass them to ecl_cc_build_csr.
+ * ecl_cc_read_mtx: MatrixMarket "coordinate" files (SMC / SuiteSparse, the source of most
+ *   of Table 2's graphs); 1-based (i, j) entries become 0-based edges, any value
+ *   columns are ignored, n = max(rows, cols).
+ * ecl_cc_read_edgelist: whitespace-separated "a b" lines, '#' or '%' comment lines (SNAP);
+ *   0-based IDs, n = 1 + the largest ID.
+ * Errors: INVALID_ARG (null argument / unreadable file), INVALID_GRAPH (malformed file or
+ * index out of range), OOM; the message is available from ecl_cc_io_last_error() (per
+ * host thread). */
+ECL_CC_API ecl_cc_status ecl_cc_read_mtx(const char *path, int32_t *n_out, int64_t *num_edges_out,
+                                         int32_t **src_out, int32_t **dst_out);
+ECL_CC_API ecl_cc_status ecl_cc_read_edgelist(const char *path, int32_t *n_out,
+                                              int64_t *num_edges_out, int32_t **src_out,
+                                              int32_t **dst_out);
+ECL_CC_API void ecl_cc_free_host(void *p);
+ECL_CC_API const char *ecl_cc_io_last_error(void);
+
 /* ---- multi-GPU building blocks (the transport is the caller's NCCL process group) ----
  * ecl_cc_run_rows: local forest of the rows [row_lo, row_hi) of a graph with n vertices.
  *   m_rows       entries of the slice (== nindex_rows[row_hi-row_lo])
@@ -149,8 +205,12 @@ typedef enum {
     ECL_CC_OPT_FINI = 13,         /* 3 = single (default), 1 = intermediate, 2 = multiple */
     ECL_CC_OPT_BATCH = 14,        /* 1 (default) = batched two-hop gathers with early exit
                                      at v_rep (R16/R19); 0 = one find per edge */
-    ECL_CC_OPT_FILTER = 15        /* anchor-tree membership bitmap (R21): 0 off,
+    ECL_CC_OPT_FILTER = 15,       /* anchor-tree membership bitmap (R21): 0 off,
                                      1 on, 2 (default) = on when 4n > 128 MB             */
+    ECL_CC_OPT_ORDER = 16         /* order of the three independent hook kernels: 0 =
+                                     thread, warp, block (paper, default); 1 =
+                                     block, warp, thread (hubs first).  Labels are the
+                                     same either way (R13).                            */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 
@@ -164,6 +224,14 @@ ECL_CC_API ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, in
  * [0] successful hook CASes, [1] failed hook CASes, [2] find_repres steps,
  * [3] path-halving stores.  Synchronises; counters reset at the start of every run. */
 ECL_CC_API ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4]);
+
+/* The same counters and the edge-filter breakdown of the batched hook path (count <= 16):
+ * [4] entries with v > u (Fig. 6 line 1), [5] of those skipped as same-tree by R15
+ * (u == parent[v] or u == v_rep), [6] checked against the R21 bitmap, [7] skipped by the
+ * bitmap, [8] hop-1 gathers parent[u], [9] hop-2 gathers, [10] bitmap marks,
+ * [11] non-empty edge windows (process_window calls), [12] edges deferred to the R22
+ * hook queue.  Others are 0. */
+ECL_CC_API ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int count);
 
 /* Per-phase device time of the most recent full run with ECL_CC_OPT_TIMING set
  * (synchronises on it): ms[0] init_bin (incl. the counter memset), ms[1] hook_thread,

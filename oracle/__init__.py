@@ -9,6 +9,10 @@ Functions (each follows the passage cited in oracle/oracle.c):
   uf(nindex, nlist)       -> (labels, ncc)   O2, P:L53 (§1) serial union-find, union by min
   init3(nindex, nlist)    -> parent          Init3, P:L141 (§3)
   check(nindex, nlist, labels, ncc) -> int   invariants I1–I3; 0 = ok
+  check_forest(nindex, nlist, labels, ta, tb) -> int   spanning-forest definition; 0 = ok
+  bfs_forest(nindex, nlist) -> (ta, tb, ncc)  the BFS tree edges of O1 (a valid forest)
+  build_csr(n, src, dst) -> (nindex, nlist)  P:L223 input preparation (loops, multi-edges,
+                                              back edges), rows ascending
 
 Inputs are numpy arrays (CSR: ``nindex`` of n+1 offsets, int32 or int64; ``nlist`` int32).
 """
@@ -67,6 +71,12 @@ def _load():
         lib.oracle_init3.restype = None
         lib.oracle_check.argtypes = [ctypes.c_int32, p, p, p, ctypes.c_int64]
         lib.oracle_check.restype = ctypes.c_int
+        lib.oracle_check_forest.argtypes = [ctypes.c_int32, p, p, p, p, p]
+        lib.oracle_check_forest.restype = ctypes.c_int
+        lib.oracle_bfs_forest.argtypes = [ctypes.c_int32, p, p, p, p]
+        lib.oracle_bfs_forest.restype = ctypes.c_int64
+        lib.oracle_build_csr.argtypes = [ctypes.c_int32, ctypes.c_int64, p, p, p, p]
+        lib.oracle_build_csr.restype = ctypes.c_int64
         _lib = lib
     return _lib
 
@@ -115,3 +125,37 @@ def check(nindex, nlist, labels, ncc_expected: int) -> int:
     if labels.shape[0] != n:
         raise ValueError("labels must have n entries")
     return int(_load().oracle_check(n, _ptr(nindex), _ptr(nlist), _ptr(labels), int(ncc_expected)))
+
+
+def check_forest(nindex, nlist, labels, ta, tb) -> int:
+    """0 if the per-vertex edge slots (ta, tb) form a spanning forest of the graph (labels =
+    the oracle's min-ID labels, which fix the (-1, -1) slots of component minima)."""
+    n, nindex, nlist = _csr(nindex, nlist)
+    arrs = [np.ascontiguousarray(np.asarray(a), dtype=np.int32) for a in (labels, ta, tb)]
+    if any(a.shape[0] != n for a in arrs):
+        raise ValueError("labels, ta and tb must have n entries")
+    return int(_load().oracle_check_forest(n, _ptr(nindex), _ptr(nlist), *(_ptr(a) for a in arrs)))
+
+
+def bfs_forest(nindex, nlist):
+    n, nindex, nlist = _csr(nindex, nlist)
+    ta = np.empty(n, dtype=np.int32)
+    tb = np.empty(n, dtype=np.int32)
+    ncc = _load().oracle_bfs_forest(n, _ptr(nindex), _ptr(nlist), _ptr(ta), _ptr(tb))
+    if ncc < 0:
+        raise MemoryError("oracle_bfs_forest failed")
+    return ta, tb, int(ncc)
+
+
+def build_csr(n: int, src, dst):
+    src = np.ascontiguousarray(np.asarray(src), dtype=np.int32)
+    dst = np.ascontiguousarray(np.asarray(dst), dtype=np.int32)
+    if src.shape != dst.shape:
+        raise ValueError("src and dst must have the same length")
+    E = src.shape[0]
+    nindex = np.empty(n + 1, dtype=np.int64)
+    nlist = np.empty(max(2 * E, 1), dtype=np.int32)
+    m = _load().oracle_build_csr(n, E, _ptr(src), _ptr(dst), _ptr(nindex), _ptr(nlist))
+    if m < 0:
+        raise ValueError("oracle_build_csr: vertex ID out of range or allocation failure")
+    return nindex, nlist[:m].copy()

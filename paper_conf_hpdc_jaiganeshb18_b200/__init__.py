@@ -24,7 +24,8 @@ import torch
 
 from . import build as _build
 
-__all__ = ["Handle", "run", "run_host", "EclCCError", "library_path", "OPT"]
+__all__ = ["Handle", "run", "run_host", "EclCCError", "library_path", "OPT", "read_mtx",
+           "read_edgelist"]
 
 OPT = {
     "thresh_thread": 1,
@@ -42,6 +43,7 @@ OPT = {
     "fini": 13,
     "batch": 14,
     "filter": 15,
+    "order": 16,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 
@@ -81,13 +83,22 @@ def _load(stats: bool = False) -> ctypes.CDLL:
             "ecl_cc_run": ([P, I32, I64, P, P, P, P], INT),
             "ecl_cc_run_i64": ([P, I32, I64, P, P, P, P], INT),
             "ecl_cc_run_host": ([P, I32, I64, P, INT, P, P, P], INT),
+            "ecl_cc_spanning_forest": ([P, I32, I64, P, INT, P, P, P, P, P], INT),
             "ecl_cc_run_rows": ([P, I32, I32, I32, I64, P, P, P, P], INT),
+            "ecl_cc_build_csr": ([P, I32, I64, P, P, P, P, I64, ctypes.POINTER(I64), P], INT),
+            "ecl_cc_read_mtx": ([ctypes.c_char_p, ctypes.POINTER(I32), ctypes.POINTER(I64),
+                                 ctypes.POINTER(P), ctypes.POINTER(P)], INT),
+            "ecl_cc_read_edgelist": ([ctypes.c_char_p, ctypes.POINTER(I32), ctypes.POINTER(I64),
+                                      ctypes.POINTER(P), ctypes.POINTER(P)], INT),
+            "ecl_cc_free_host": ([P], None),
+            "ecl_cc_io_last_error": ([], ctypes.c_char_p),
             "ecl_cc_merge": ([P, I32, I32, I32, P, P, P], INT),
             "ecl_cc_finalize": ([P, I32, P, P], INT),
             "ecl_cc_validate": ([P, I32, I64, P, INT, P, P], INT),
             "ecl_cc_set_option": ([P, INT, I64], INT),
             "ecl_cc_get_worklist": ([P, P, ctypes.POINTER(I64), P, ctypes.POINTER(I64)], INT),
             "ecl_cc_get_stats": ([P, ctypes.POINTER(I64)], INT),
+            "ecl_cc_get_stats_ex": ([P, ctypes.POINTER(I64), INT], INT),
             "ecl_cc_stats_enabled": ([], INT),
             "ecl_cc_get_timing": ([P, ctypes.POINTER(ctypes.c_float)], INT),
             "ecl_cc_status_string": ([INT], ctypes.c_char_p),
@@ -192,6 +203,43 @@ class Handle:
                        _stream_ptr(stream, d)))
         return out
 
+    def spanning_forest(self, nindex: torch.Tensor, nlist: torch.Tensor, stream=None):
+        """(labels, tree_a, tree_b): min-ID labels and, for every vertex x that is not its
+        component's minimum, a CSR edge (tree_a[x], tree_b[x]); together these edges form a
+        spanning forest (ecl_cc_spanning_forest).  Entries of component minima are -1."""
+        d = self.device
+        _dev_tensor(nindex, "nindex", (torch.int32, torch.int64), d)
+        _dev_tensor(nlist, "nlist", (torch.int32,), d)
+        n = nindex.numel() - 1
+        if n < 0:
+            raise ValueError("nindex must hold n+1 offsets")
+        labels = torch.empty(n, dtype=torch.int32, device=d)
+        ta = torch.empty(n, dtype=torch.int32, device=d)
+        tb = torch.empty(n, dtype=torch.int32, device=d)
+        self._check(self._lib.ecl_cc_spanning_forest(
+            self._h, n, nlist.numel(), _ptr(nindex), nindex.element_size(), _ptr(nlist),
+            _ptr(labels), _ptr(ta), _ptr(tb), _stream_ptr(stream, d)))
+        return labels, ta, tb
+
+    def build_csr(self, n: int, src: torch.Tensor, dst: torch.Tensor, stream=None):
+        """(nindex int64[n+1], nlist int32[m]) on the device: the symmetric, loop-free,
+        duplicate-free CSR of the undirected edge list (src[i], dst[i]) (ecl_cc_build_csr,
+        P:L223).  Synchronises the stream."""
+        d = self.device
+        _dev_tensor(src, "src", (torch.int32,), d)
+        _dev_tensor(dst, "dst", (torch.int32,), d)
+        if src.numel() != dst.numel():
+            raise ValueError("src and dst must have the same length")
+        E = src.numel()
+        nindex = torch.empty(n + 1, dtype=torch.int64, device=d)
+        cap = max(2 * E, 1)
+        nlist = torch.empty(cap, dtype=torch.int32, device=d)
+        m = ctypes.c_int64(0)
+        self._check(self._lib.ecl_cc_build_csr(self._h, n, E, _ptr(src), _ptr(dst), _ptr(nindex),
+                                               _ptr(nlist), cap, ctypes.byref(m),
+                                               _stream_ptr(stream, d)))
+        return nindex, nlist[:m.value].clone()
+
     def run_host(self, nindex, nlist, out=None, stream=None):
         """End-to-end on host buffers (numpy arrays or CPU tensors, ideally pinned)."""
         import numpy as np
@@ -275,11 +323,16 @@ class Handle:
         self._check(self._lib.ecl_cc_get_timing(self._h, arr))
         return dict(zip(PHASES, list(arr)))
 
+    STAT_NAMES = ("cas_success", "cas_fail", "finds", "halving_stores", "edges_v_gt_u",
+                  "edges_r15_same_tree", "edges_bitmap_checked", "edges_bitmap_skipped",
+                  "gathers_hop1", "gathers_hop2", "bitmap_marks", "windows", "edges_queued")
+
     def stats(self) -> dict:
-        arr = (ctypes.c_int64 * 4)()
-        self._check(self._lib.ecl_cc_get_stats(self._h, arr))
-        return {"cas_success": arr[0], "cas_fail": arr[1], "finds": arr[2],
-                "halving_stores": arr[3]}
+        """ECL_CC_STATS counters of the last run (ecl_cc_get_stats_ex)."""
+        k = len(self.STAT_NAMES)
+        arr = (ctypes.c_int64 * k)()
+        self._check(self._lib.ecl_cc_get_stats_ex(self._h, arr, k))
+        return dict(zip(self.STAT_NAMES, list(arr)))
 
 
 _default = {}
@@ -301,3 +354,35 @@ def run(nindex: torch.Tensor, nlist: torch.Tensor, out: Optional[torch.Tensor] =
 def run_host(nindex, nlist, out=None, device=None):
     """End-to-end on host arrays: H2D copy, run, D2H copy (synchronous)."""
     return _handle(device).run_host(nindex, nlist, out=out)
+
+
+def _read(fn_name: str, path: str):
+    import numpy as np
+    lib = _load()
+    n = ctypes.c_int32(0)
+    e = ctypes.c_int64(0)
+    a = ctypes.c_void_p()
+    b = ctypes.c_void_p()
+    st = getattr(lib, fn_name)(os.fsencode(path), ctypes.byref(n), ctypes.byref(e),
+                               ctypes.byref(a), ctypes.byref(b))
+    if st != 0:
+        raise EclCCError(st, lib.ecl_cc_io_last_error().decode())
+    try:
+        k = e.value
+        src = np.ctypeslib.as_array((ctypes.c_int32 * max(k, 1)).from_address(a.value))[:k].copy()
+        dst = np.ctypeslib.as_array((ctypes.c_int32 * max(k, 1)).from_address(b.value))[:k].copy()
+    finally:
+        lib.ecl_cc_free_host(a)
+        lib.ecl_cc_free_host(b)
+    return n.value, src, dst
+
+
+def read_mtx(path: str):
+    """(n, src, dst) numpy int32 edge list of a MatrixMarket coordinate file (ecl_cc_read_mtx;
+    host-only C reader, no GPU needed)."""
+    return _read("ecl_cc_read_mtx", path)
+
+
+def read_edgelist(path: str):
+    """(n, src, dst) of a SNAP-style whitespace edge list (ecl_cc_read_edgelist)."""
+    return _read("ecl_cc_read_edgelist", path)

@@ -13,8 +13,10 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-SOURCES = [os.path.join(CSRC, "ecl_cc.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, "ecl_cc_kernels.cuh"), os.path.join(INCLUDE, "ecl_cc.h")]
+SOURCES = [os.path.join(CSRC, "ecl_cc.cu"), os.path.join(CSRC, "ecl_cc_csr.cu"),
+           os.path.join(CSRC, "ecl_cc_io.cpp")]
+DEPS = SOURCES + [os.path.join(CSRC, "ecl_cc_kernels.cuh"), os.path.join(CSRC, "ecl_cc_ctx.h"),
+                  os.path.join(INCLUDE, "ecl_cc.h")]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -5,6 +5,7 @@
 //   -> finalize, all enqueued on the caller's stream with no host synchronisation.
 #include "ecl_cc.h"
 #include "ecl_cc_kernels.cuh"
+#include "ecl_cc_ctx.h"
 
 #include <algorithm>
 #include <cstdio>
@@ -13,83 +14,15 @@
 #include <unordered_map>
 
 using namespace eclcc;
-
-struct ecl_cc_ctx {
-    int device = 0;
-    int sms = 0;
-    // scratch (device, grow-only)
-    int *wl = nullptr;
-    unsigned *ub = nullptr;
-    int cap = 0;
-    unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [2..5] stats,
-                                          // [8..9] int scheduling counters
-    int *flags = nullptr;                 // validate flags
-    // end-to-end buffers (device, grow-only)
-    void *e2e_index = nullptr;
-    size_t e2e_index_bytes = 0;
-    int *e2e_list = nullptr;
-    size_t e2e_list_n = 0;
-    int *e2e_labels = nullptr;
-    size_t e2e_labels_n = 0;
-    // options
-    int t1 = 16, t2 = 352;
-    int grid_blocks = 0;
-    int occ_thread = 0, occ_range = 0;    // blocks per SM caps (0 = max occupancy)
-    int init_mode = 3, jump = 4, fini = 3; // paper ablation variants (defaults = ECL-CC)
-    int batch = 1;                        // batched two-hop gathers (R16, R19)
-    int filter = 2;                       // R21 membership filter: 0 off, 1 on, 2 auto
-    unsigned *gbits = nullptr;            // R21 bitmap (grow-only)
-    size_t gbits_words = 0;
-    int stop_after = 0;
-    int load_mode = 1;
-    int ttas = 1;                         // test-and-test-and-set hooks
-    int timing = 0;                       // record per-kernel CUDA events
-    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
-    int ev_valid = 0;
-    // last run (for ecl_cc_get_worklist)
-    cudaStream_t last_stream = nullptr;
-    std::unordered_map<const void *, int> occ;
-    char err[512] = {0};
-};
+using namespace eclcc_host;
 
 namespace {
 
+constexpr int kCnt = 32;        // 64-bit counter words owned by the handle
+constexpr int kStatsOff = 16;   // ECL_CC_STATS counters live at cnt[16..31]
+constexpr int kNumStats = 16;
+
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
-
-ecl_cc_status fail_cuda(ecl_cc_handle h, cudaError_t e, const char *where)
-{
-    if (h) snprintf(h->err, sizeof(h->err), "%s: %s (%s)", where, cudaGetErrorString(e),
-                    cudaGetErrorName(e));
-    return e == cudaErrorMemoryAllocation ? ECL_CC_ERR_OOM : ECL_CC_ERR_CUDA;
-}
-
-ecl_cc_status fail_arg(ecl_cc_handle h, const char *msg)
-{
-    if (h) snprintf(h->err, sizeof(h->err), "invalid argument: %s", msg);
-    return ECL_CC_ERR_INVALID_ARG;
-}
-
-#define CK(call, where)                                      \
-    do {                                                     \
-        cudaError_t e_ = (call);                             \
-        if (e_ != cudaSuccess) return fail_cuda(h, e_, where); \
-    } while (0)
-
-// Make `dev` current for the duration of a call, restoring the caller's device.
-struct DeviceGuard {
-    int prev = -1;
-    bool ok = true;
-    explicit DeviceGuard(int dev)
-    {
-        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
-        if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
-    }
-    ~DeviceGuard()
-    {
-        int cur = -1;
-        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
-    }
-};
 
 int blocks_per_sm(ecl_cc_handle h, const void *kernel, size_t dsmem)
 {
@@ -140,7 +73,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
 {
     ecl_cc_status st = ensure_scratch(h, nrows > 0 ? nrows : 1, s);
     if (st != ECL_CC_OK) return st;
-    CK(cudaMemsetAsync(h->cnt, 0, 16 * sizeof(unsigned long long), s), "cudaMemsetAsync");
+    CK(cudaMemsetAsync(h->cnt, 0, kCnt * sizeof(unsigned long long), s), "cudaMemsetAsync");
     h->last_stream = s;
 
     Params p;
@@ -155,7 +88,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.ub = h->ub;
     p.cap = h->cap;
     p.cnt = h->cnt;
-    p.stats = h->cnt + 2;
+    p.stats = h->cnt + kStatsOff;
     p.sched = (int *)(h->cnt + 8);
     p.t1 = h->t1;
     p.t2 = h->t2;
@@ -165,6 +98,8 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.batch = h->batch;
     p.anchor = h->cnt + 10;
     p.gbits = nullptr;
+    p.fa = h->fa;
+    p.fb = h->fb;
     {
         // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
         const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
@@ -202,31 +137,45 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     }
     mark(1);
     if (h->stop_after != 1) {
-        {
+        // the three compute kernels depend only on init_bin; events record each
+        // kernel's span whatever the launch order (ev[2+i] ends phase i)
+        auto thread_k = [&] {
             auto k = hook_thread_kernel<MODE, idx_t>;
             const long long tiles = (nrows + kWarp - 1) / kWarp;
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, tiles * kWarp, sm, h->occ_thread), kBlock, sm, s>>>(p);
-        }
-        mark(2);
-        {
+        };
+        auto warp_k = [&] {
             auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
-        }
-        mark(3);
-        {
+        };
+        auto block_k = [&] {
             auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
+        };
+        if (h->order == 1) {
+            block_k();
+            mark(4);
+            warp_k();
+            mark(3);
+            thread_k();
+            mark(2);
+        } else {
+            thread_k();
+            mark(2);
+            warp_k();
+            mark(3);
+            block_k();
+            mark(4);
         }
-        mark(4);
         if (h->stop_after != 2) {
             auto k = finalize_kernel<MODE>;
             k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
         }
         mark(5);
-        if (tm && h->stop_after == 0) h->ev_valid = 1;
+        if (tm && h->stop_after == 0) h->ev_valid = 1 + h->order;
     }
     CK(cudaGetLastError(), "kernel launch");
     return ECL_CC_OK;
@@ -273,7 +222,7 @@ ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device)
     h->device = device;
     DeviceGuard g(device);
     cudaError_t e = cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, 16 * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, kCnt * sizeof(unsigned long long));
     if (e == cudaSuccess) e = cudaMalloc((void **)&h->flags, 4 * sizeof(int));
     if (e != cudaSuccess) {
         if (h->cnt) cudaFree(h->cnt);
@@ -298,6 +247,7 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
         if (h->e2e_list) cudaFree(h->e2e_list);
         if (h->e2e_labels) cudaFree(h->e2e_labels);
         if (h->gbits) cudaFree(h->gbits);
+        if (h->csr_tmp) cudaFree(h->csr_tmp);
         for (int i = 0; i < 6; i++)
             if (h->ev[i]) cudaEventDestroy(h->ev[i]);
     }
@@ -317,6 +267,25 @@ ecl_cc_status ecl_cc_run_i64(ecl_cc_handle h, int32_t n, int64_t m, const int64_
 {
     return run_impl<long long>(h, n, m, (const long long *)nindex, nlist, nstat_out, stream, 0,
                                n, false);
+}
+
+ecl_cc_status ecl_cc_spanning_forest(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex,
+                                     int index_bytes, const int32_t *nlist,
+                                     int32_t *labels_out, int32_t *tree_a, int32_t *tree_b,
+                                     void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (index_bytes != 4 && index_bytes != 8) return fail_arg(h, "index_bytes must be 4 or 8");
+    if (n > 0 && (!tree_a || !tree_b)) return fail_arg(h, "null tree-edge output");
+    if (h->stop_after != 0) return fail_arg(h, "spanning forest needs a full run (stop_after 0)");
+    h->fa = tree_a;
+    h->fb = tree_b;
+    ecl_cc_status st = index_bytes == 4
+        ? ecl_cc_run(h, n, m, (const int32_t *)nindex, nlist, labels_out, stream)
+        : ecl_cc_run_i64(h, n, m, (const int64_t *)nindex, nlist, labels_out, stream);
+    h->fa = nullptr;
+    h->fb = nullptr;
+    return st;
 }
 
 ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
@@ -343,14 +312,14 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
         auto k = merge_hook_kernel<1>;
         k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
-                                                                 , h->cnt + 2
+                                                                 , h->cnt + kStatsOff
 #endif
         );
     } else {
         auto k = merge_hook_kernel<0>;
         k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
-                                                                 , h->cnt + 2
+                                                                 , h->cnt + kStatsOff
 #endif
         );
     }
@@ -521,6 +490,10 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         if (value < 0 || value > 2) return fail_arg(h, "filter must be 0, 1 or 2");
         h->filter = (int)value;
         break;
+    case ECL_CC_OPT_ORDER:
+        if (value < 0 || value > 1) return fail_arg(h, "order must be 0 or 1");
+        h->order = (int)value;
+        break;
     case ECL_CC_OPT_BATCH:
         h->batch = value != 0;
         break;
@@ -562,15 +535,20 @@ ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, int64_t *nfro
     return ECL_CC_OK;
 }
 
+ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int count)
+{
+    if (!h || !out || count < 0 || count > kNumStats) return ECL_CC_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
+    unsigned long long c[kNumStats] = {};
+    CK(cudaStreamSynchronize(h->last_stream), "sync");
+    CK(cudaMemcpy(c, h->cnt + kStatsOff, sizeof(c), cudaMemcpyDeviceToHost), "D2H stats");
+    for (int i = 0; i < count; i++) out[i] = (int64_t)c[i];
+    return ECL_CC_OK;
+}
+
 ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4])
 {
-    if (!h || !out) return ECL_CC_ERR_INVALID_ARG;
-    DeviceGuard g(h->device);
-    unsigned long long c[4] = {0, 0, 0, 0};
-    CK(cudaStreamSynchronize(h->last_stream), "sync");
-    CK(cudaMemcpy(c, h->cnt + 2, sizeof(c), cudaMemcpyDeviceToHost), "D2H stats");
-    for (int i = 0; i < 4; i++) out[i] = (int64_t)c[i];
-    return ECL_CC_OK;
+    return ecl_cc_get_stats_ex(h, out, 4);
 }
 
 ecl_cc_status ecl_cc_get_timing(ecl_cc_handle h, float ms[5])
@@ -579,7 +557,11 @@ ecl_cc_status ecl_cc_get_timing(ecl_cc_handle h, float ms[5])
     if (!h->ev_valid) return fail_arg(h, "no timed full run recorded (set ECL_CC_OPT_TIMING)");
     DeviceGuard g(h->device);
     CK(cudaEventSynchronize(h->ev[5]), "cudaEventSynchronize");
-    for (int i = 0; i < 5; i++) CK(cudaEventElapsedTime(&ms[i], h->ev[i], h->ev[i + 1]), "elapsed");
+    // phase i spans ev[from[i]] -> ev[to[i]] (the hook kernels may run in reverse order)
+    static const int from0[5] = {0, 1, 2, 3, 4}, to0[5] = {1, 2, 3, 4, 5};
+    static const int from1[5] = {0, 3, 4, 1, 2}, to1[5] = {1, 2, 3, 4, 5};
+    const int *from = h->ev_valid == 2 ? from1 : from0, *to = h->ev_valid == 2 ? to1 : to0;
+    for (int i = 0; i < 5; i++) CK(cudaEventElapsedTime(&ms[i], h->ev[from[i]], h->ev[to[i]]), "elapsed");
     return ECL_CC_OK;
 }
 

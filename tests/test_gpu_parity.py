@@ -317,3 +317,64 @@ def test_membership_filter(h, name, grid):
 def test_load_modes_with_filter(h, mode):
     g = gg.make_config("C5", seed=9, scale_down=9, device="cuda")
     assert_parity(h, g, filter=1, load_mode=mode)
+
+
+# ---------------------------------------------------------------------------------------
+# kernel order option (hubs first): same labels
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", list(SMALL))
+def test_order_hubs_first(h, name):
+    g = gg.make_config(name, seed=12, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, order=1)
+    assert_parity(h, g, order=1, filter=1)
+
+
+# ---------------------------------------------------------------------------------------
+# spanning forest: labels bit-exact, forest valid by the oracle's checker
+# (the forest itself is one of many valid answers)
+# ---------------------------------------------------------------------------------------
+def assert_forest(h, g, index_dtype=None, **opts):
+    g = g.to("cuda")
+    nindex = g.nindex if index_dtype is None else g.nindex.to(index_dtype)
+    for k, v in opts.items():
+        h.set_option(k, v)
+    try:
+        lab, ta, tb = h.spanning_forest(nindex, g.nlist)
+        torch.cuda.synchronize()
+    finally:
+        for k in opts:
+            h.set_option(k, DEFAULTS.get(k, 0))
+    nidx, nl = g.numpy()
+    expect, ncc = oracle.bfs(nidx, nl)
+    lab = lab.cpu().numpy()
+    assert np.array_equal(lab, expect), f"{g.name}: labels differ"
+    rc = oracle.check_forest(nidx, nl, expect, ta.cpu().numpy(), tb.cpu().numpy())
+    assert rc == 0, f"{g.name}: forest check failed with code {rc}"
+
+
+@pytest.mark.parametrize("g", hand_graphs(), ids=lambda g: g.name)
+def test_forest_hand_built(h, g):
+    assert_forest(h, g)
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("seed", [1, 2])
+def test_forest_configs(h, name, seed):
+    g = gg.make_config(name, seed=seed, scale_down=SMALL[name], device="cuda")
+    assert_forest(h, g)
+    assert_forest(h, gg.shuffle_rows(g, seed=seed + 10))
+
+
+@pytest.mark.parametrize("opts", [dict(filter=1), dict(order=1), dict(ttas=0),
+                                  dict(init=1), dict(init=2), dict(jump=1), dict(jump=3),
+                                  dict(batch=0), dict(grid_blocks=3), dict(load_mode=0)],
+                         ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
+def test_forest_variants(h, opts):
+    g = gg.make_config("C4", seed=5, scale_down=8, device="cuda")
+    assert_forest(h, g, **opts)
+    assert_forest(h, gg.make_config("C2", seed=5, scale_down=6, device="cuda"), **opts)
+
+
+def test_forest_int64_offsets(h):
+    g = gg.make_config("C5", seed=4, scale_down=9, device="cuda")
+    assert_forest(h, g, index_dtype=torch.int64)

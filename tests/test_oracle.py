@@ -200,3 +200,146 @@ def test_table2_r4_statistical_small():
     _, ncc = oracle.bfs(*g.numpy())
     assert ncc == 1
     assert int(d.min()) >= 4 and abs(float(d.double().mean()) - 8.0) < 0.01
+
+
+# ---- spanning-forest checker (oracle_check_forest) ----------------------
+
+def _slots(n, labels, edges, rng):
+    """Assign a list of undirected edges to the non-minimum vertices' slots (the CUDA
+    path's output format), each edge in a random orientation; minima get (-1, -1)."""
+    ta = np.full(n, -1, dtype=np.int32)
+    tb = np.full(n, -1, dtype=np.int32)
+    slots = [x for x in range(n) if labels[x] != x]
+    assert len(slots) == len(edges)
+    for x, (a, b) in zip(slots, edges):
+        if rng.random() < 0.5:
+            a, b = b, a
+        ta[x], tb[x] = a, b
+    return ta, tb
+
+
+def _closure_classes(n, edges):
+    adj = np.zeros((1, n, n), dtype=bool)
+    for a, b in edges:
+        adj[0, a, b] = adj[0, b, a] = True
+    return len(set(closure_labels(adj)[0].tolist()))
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5])
+def test_forest_checker_brute_force(n):
+    """Every subset S of a graph's edges with |S| = n - #CC is fed to the checker; it must
+    accept exactly the subsets whose transitive closure has #CC classes (brute force)."""
+    rng = np.random.default_rng(n)
+    pairs = list(itertools.combinations(range(n), 2))
+    graphs = range(1 << len(pairs))
+    if n == 5:
+        graphs = rng.choice(1 << len(pairs), 150, replace=False)
+    for g in graphs:
+        edges = [pairs[k] for k in range(len(pairs)) if (int(g) >> k) & 1]
+        nindex, nlist = csr_np(n, edges)
+        labels, ncc = oracle.bfs(nindex, nlist)
+        for S in itertools.combinations(edges, n - ncc):
+            ta, tb = _slots(n, labels, list(S), rng)
+            spans = _closure_classes(n, S) == ncc
+            rc = oracle.check_forest(nindex, nlist, labels, ta, tb)
+            assert rc == (0 if spans else 3), (n, edges, S, rc)
+
+
+def test_forest_checker_mutations():
+    g = gg.erdos_renyi(3000, 4000, seed=5)
+    nindex, nlist = g.numpy()
+    labels, ncc = oracle.bfs(nindex, nlist)
+    ta, tb, ncc2 = oracle.bfs_forest(nindex, nlist)
+    assert ncc2 == ncc
+    assert oracle.check_forest(nindex, nlist, labels, ta, tb) == 0
+    non_min = np.flatnonzero(labels != np.arange(g.n))
+    x = int(non_min[7])
+    # a pair that is not a CSR entry
+    a, b = ta.copy(), tb.copy()
+    row = set(nlist[nindex[a[x]]:nindex[a[x] + 1]].tolist())
+    b[x] = next(w for w in range(g.n) if w not in row and w != a[x])
+    assert oracle.check_forest(nindex, nlist, labels, a, b) == 2
+    # out of range
+    a, b = ta.copy(), tb.copy()
+    b[x] = g.n
+    assert oracle.check_forest(nindex, nlist, labels, a, b) == 2
+    # a non-minimum slot left empty / a minimum slot filled
+    a, b = ta.copy(), tb.copy()
+    a[x] = b[x] = -1
+    assert oracle.check_forest(nindex, nlist, labels, a, b) == 1
+    a, b = ta.copy(), tb.copy()
+    mn = int(np.flatnonzero(labels == np.arange(g.n))[0])
+    a[mn], b[mn] = ta[x], tb[x]
+    assert oracle.check_forest(nindex, nlist, labels, a, b) == 1
+    # a duplicated tree edge: some slot repeats another slot's edge -> cycle (2-cycle)
+    a, b = ta.copy(), tb.copy()
+    y = int(non_min[8])
+    a[y], b[y] = tb[x], ta[x]
+    assert oracle.check_forest(nindex, nlist, labels, a, b) == 3
+
+
+def test_forest_checker_accepts_scipy_spanning_trees():
+    """scipy's minimum_spanning_tree (Kruskal) of random weighted graphs is a spanning
+    forest by a library routine independent of the oracle."""
+    from scipy.sparse import csr_matrix
+    from scipy.sparse.csgraph import minimum_spanning_tree
+    rng = np.random.default_rng(77)
+    for trial in range(40):
+        n = int(rng.integers(2, 600))
+        m = int(rng.integers(0, 2 * n))
+        pairs = {(int(min(a, b)), int(max(a, b))) for a, b in
+                 zip(rng.integers(0, n, m), rng.integers(0, n, m)) if a != b}
+        nindex, nlist = csr_np(n, sorted(pairs))
+        labels, ncc = oracle.bfs(nindex, nlist)
+        w = rng.random(len(nlist)) + 1.0
+        rows = np.repeat(np.arange(n), np.diff(nindex))
+        W = {}
+        for r, c, x in zip(rows, nlist, w):
+            W[(min(r, c), max(r, c))] = x
+        keys = sorted(W)
+        A = csr_matrix(([W[k] for k in keys], ([k[0] for k in keys], [k[1] for k in keys])),
+                       shape=(n, n))
+        T = minimum_spanning_tree(A).tocoo()
+        edges = list(zip(T.row.tolist(), T.col.tolist()))
+        assert len(edges) == n - ncc
+        ta, tb = _slots(n, labels, edges, rng)
+        assert oracle.check_forest(nindex, nlist, labels, ta, tb) == 0
+
+
+# ---- CSR preparation (oracle_build_csr) -----------------------------------------
+
+def test_build_csr_hand_examples():
+    # loops dropped, duplicates merged (both orientations), back edges added, rows sorted
+    nindex, nlist = oracle.build_csr(5, [3, 1, 1, 2, 3, 4], [1, 3, 1, 0, 1, 4])
+    assert nindex.tolist() == [0, 1, 2, 3, 4, 4]
+    assert nlist.tolist() == [2, 3, 0, 1]
+    nindex, nlist = oracle.build_csr(3, [], [])
+    assert nindex.tolist() == [0, 0, 0, 0] and nlist.size == 0
+    with pytest.raises(ValueError):
+        oracle.build_csr(3, [0], [3])
+
+
+def test_build_csr_matches_scipy():
+    """scipy: A = coo(1) + its transpose, diagonal removed, duplicates summed then binarised,
+    canonical (sorted) CSR — a library route independent of the oracle's qsort."""
+    from scipy.sparse import coo_matrix
+    rng = np.random.default_rng(99)
+    for trial in range(60):
+        n = int(rng.integers(1, 3000))
+        E = int(rng.integers(0, 4 * n))
+        a = rng.integers(0, n, E).astype(np.int32)
+        b = rng.integers(0, n, E).astype(np.int32)
+        if trial % 3 == 0 and E >= 4:     # extra loops and duplicates
+            q = E // 4
+            a[:q] = b[:q]                     # loops
+            a[q:2 * q] = b[2 * q:3 * q]       # reversed duplicates of later pairs
+            b[q:2 * q] = a[2 * q:3 * q]
+        nindex, nlist = oracle.build_csr(n, a, b)
+        A = coo_matrix((np.ones(E), (a, b)), shape=(n, n)).tocsr()
+        A = (A + A.T).tolil()
+        A.setdiag(0)
+        A = A.tocsr()
+        A.eliminate_zeros()
+        A.sort_indices()
+        assert np.array_equal(nindex, A.indptr.astype(np.int64))
+        assert np.array_equal(nlist, A.indices.astype(np.int32))
