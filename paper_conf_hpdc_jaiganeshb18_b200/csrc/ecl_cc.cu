@@ -97,6 +97,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.jump = h->jump;
     p.batch = h->batch;
     p.anchor = h->cnt + 10;
+    p.nthr = h->cnt + 3;
     p.gbits = nullptr;
     p.fa = h->fa;
     p.fb = h->fb;

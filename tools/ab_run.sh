@@ -11,7 +11,7 @@ for c in $CFGS; do
     v=${spec%%@*}; a=""
     [[ "$spec" == *@* ]] && a=${spec#*@}
     echo -n "{\"variant\": \"$spec\", \"r\": "
-    ECL_CC_LIB=build/ab/$v.so timeout 300 python tools/prof.py --config $c --reps 5 ${a//,/ } 2>&1 | tail -1
+    ECL_CC_LIB=build/ab/$v.so timeout 300 python tools/prof.py --config $c --reps 10 ${a//,/ } 2>&1 | tail -1
     echo "}"
   done
 done > gpurun_out/ab_$TAG.jsonl

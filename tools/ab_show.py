@@ -5,7 +5,11 @@ import sys
 
 txt = open(sys.argv[1]).read()
 for blob in re.findall(r'\{"variant".*?\n\}', txt, re.S):
-    d = json.loads(blob.replace("\n", " "))
+    try:
+        d = json.loads(blob.replace("\n", " "))
+    except json.JSONDecodeError:
+        print("unparsable:", blob[:120].replace("\n", " "))
+        continue
     r = d["r"]
     b = r["best_ms"]
     print(f"{r['config']} {d['variant']:12s} total={b['total']:7.3f} init={b['init_bin']:.3f} "

@@ -10,8 +10,11 @@ KEYS = ["Duration", "DRAM Throughput", "L1/TEX Hit Rate", "L2 Hit Rate", "Memory
         "Executed Instructions", "Avg. Active Threads Per Warp"]
 
 
+KFILTER = []
+
+
 def run(args):
-    return subprocess.run(["ncu", "-i"] + args, capture_output=True, text=True).stdout
+    return subprocess.run(["ncu", "-i"] + args + KFILTER, capture_output=True, text=True).stdout
 
 
 def main(rep, top=25):
@@ -65,4 +68,7 @@ def main(rep, top=25):
         print(f"{100*s/tot:5.1f}%  inst={e:12.0f}  L{ln:>4}  {code.get(ln, '').strip()[:90]}")
 
 if __name__ == "__main__":
+    # python tools/ncu_summary.py REPORT [TOP] [KERNEL_REGEX]
+    if len(sys.argv) > 3:
+        KFILTER[:] = ["-k", "regex:" + sys.argv[3]]
     main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 25)
