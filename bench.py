@@ -198,11 +198,36 @@ def cpu_oracle_sample(config: str, seed: int, budget_s: float = 15.0):
         dt += time.perf_counter() - t1
         reps += 1
     m = int(nl.shape[0])
-    return {"value": round(m * reps / dt / 1e6, 3), "unit": "Medges/s", "cores": 1,
-            "kind": "oracle",
-            "sample": f"{config} recipe at 1/2^{sd} scale (n={nidx.shape[0]-1}, m={m}), "
-                      f"O1 serial BFS, {reps} run(s), {dt:.2f} s, single thread of "
-                      f"{os.cpu_count()} host cores"}
+    out = {"value": round(m * reps / dt / 1e6, 3), "unit": "Medges/s", "cores": 1,
+           "kind": "oracle",
+           "sample": f"{config} recipe at 1/2^{sd} scale (n={nidx.shape[0]-1}, m={m}), "
+                     f"O1 serial BFS, {reps} run(s), {dt:.2f} s, single thread of "
+                     f"{os.cpu_count()} host cores"}
+    return out, (nidx, nl)
+
+
+def cpu_paper_codes(nidx, nl, budget_s: float = 10.0):
+    """The paper's own CPU versions (ECL-CCOMP on all host cores, ECL-CCSER on one; P:L183,
+    P:L185; baselines/) on the same bounded sample as cpu_baseline: context, not the
+    oracle."""
+    import baselines
+    baselines.build()
+    m = int(nl.shape[0])
+    res = {}
+    for name, fn, cores in (("ecl_cc_omp", lambda: baselines.omp(nidx, nl), os.cpu_count()),
+                            ("ecl_cc_ser", lambda: baselines.ser(nidx, nl), 1)):
+        fn()
+        t0 = time.perf_counter()
+        reps = 0
+        while True:
+            fn()
+            reps += 1
+            if time.perf_counter() - t0 > budget_s / 4 or reps >= 5:
+                break
+        dt = time.perf_counter() - t0
+        res[name] = {"value": round(m * reps / dt / 1e6, 3), "unit": "Medges/s",
+                     "cores": cores, "runs": reps}
+    return res
 
 
 def run_reference(args):
@@ -386,8 +411,11 @@ def main():
                 "path_alg_bytes": int(b_alg),
                 "path_frac": round(b_alg / (ms_step * 1e-3) / 1e9 / peak, 4)}
     cpu = None
+    cpu_paper = None
     if world == 1 and not args.no_cpu:
-        cpu = cpu_oracle_sample(args.config, args.seed)
+        cpu, sample = cpu_oracle_sample(args.config, args.seed)
+        cpu_paper = cpu_paper_codes(*sample)
+        del sample
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "Medges/s", "n_gpus": world,
@@ -406,6 +434,7 @@ def main():
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},
         "cpu_baseline": cpu,
+        "cpu_paper_codes": cpu_paper,
         "e2e": e2e,
         "parity": ok,
         "per_step_ms": [round(x, 4) for x in per],

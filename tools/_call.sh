@@ -1,4 +1,5 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -2 gpurun_out/pytest_gpu.log
-bash tools/ab_run.sh auto "C5 C4 C3 C2" prev auto always prev auto > /dev/null
+timeout 300 python tools/l2_ceiling.py > gpurun_out/l2_ceiling.json 2>&1; cat gpurun_out/l2_ceiling.json
+timeout 600 python bench.py > gpurun_out/bench_C5.json 2> gpurun_out/bench_C5.err; echo "bench rc=$?"
+bash tools/gpu_profile.sh r1c > gpurun_out/r1c_profile.log 2>&1
