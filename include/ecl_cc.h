@@ -207,10 +207,16 @@ typedef enum {
                                      at v_rep (R16/R19); 0 = one find per edge */
     ECL_CC_OPT_FILTER = 15,       /* anchor-tree membership bitmap (R21): 0 off,
                                      1 on, 2 (default) = on when 4n > 128 MB             */
-    ECL_CC_OPT_ORDER = 16         /* order of the three independent hook kernels: 0 =
+    ECL_CC_OPT_ORDER = 16,        /* order of the three independent hook kernels: 0 =
                                      thread, warp, block (paper, default); 1 =
                                      block, warp, thread (hubs first).  Labels are the
                                      same either way (R13).                            */
+    ECL_CC_OPT_PREJUMP = 17       /* pointer-doubling passes between init and the hook
+                                     kernels (R23; Jump's pointer jumping,
+                                     P:L245, as synchronous passes): 0 off, 1 always,
+                                     2 (default) only when a sample of the Init3
+                                     forest is deep (meshes, road-like graphs).
+                                     Labels are unchanged (R13).                       */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

@@ -44,6 +44,7 @@ OPT = {
     "batch": 14,
     "filter": 15,
     "order": 16,
+    "prejump": 17,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

@@ -1,7 +1,8 @@
 // ecl_cc.cu — host side of libecl_cc.so: the C ABI declared in include/ecl_cc.h.
 //
 // Launch sequence of one run (init, three compute kernels, finalize):
-//   memset(counters) -> init_bin -> hook_thread -> hook_range<front> -> hook_range<back>
+//   memset(counters) -> init_bin -> depth_probe -> prejump (R23, no-op unless deep)
+//   -> hook_thread -> hook_range<front> -> hook_range<back>
 //   -> finalize, all enqueued on the caller's stream with no host synchronisation.
 #include "ecl_cc.h"
 #include "ecl_cc_kernels.cuh"
@@ -135,6 +136,20 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     {
         auto k = init_bin_kernel<idx_t>;
         k<<<grid_for(h, (const void *)k, ((long long)nrows + kInitPerThread - 1) / kInitPerThread), kBlock, 0, s>>>(p);
+    }
+    if (h->prejump != 0 && h->stop_after != 1 && nrows > 0) {
+        // R23: depth probe, then the passes (cooperative launch guarantees the
+        // co-residency their grid barrier needs); both are no-ops on shallow forests
+        int *ctl = (int *)(h->cnt + 4);
+        depth_probe_kernel<<<1, kBlock, 0, s>>>(row_lo, nrows, parent, ctl, h->prejump);
+        auto k = prejump_kernel;
+        const int blocks = std::min(h->sms * blocks_per_sm(h, (const void *)k, 0),
+                                    (int)std::max(1LL, ((long long)nrows + kBlock - 1) / kBlock));
+        int a0 = row_lo, a1 = nrows;
+        int *a2 = parent, *a3 = ctl;
+        void *args[] = {&a0, &a1, &a2, &a3};
+        CK(cudaLaunchCooperativeKernel((const void *)k, dim3(blocks), dim3(kBlock), args, 0, s),
+           "prejump launch");
     }
     mark(1);
     if (h->stop_after != 1) {
@@ -494,6 +509,10 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_ORDER:
         if (value < 0 || value > 1) return fail_arg(h, "order must be 0 or 1");
         h->order = (int)value;
+        break;
+    case ECL_CC_OPT_PREJUMP:
+        if (value < 0 || value > 2) return fail_arg(h, "prejump must be 0, 1 or 2");
+        h->prejump = (int)value;
         break;
     case ECL_CC_OPT_BATCH:
         h->batch = value != 0;

@@ -35,6 +35,7 @@ struct ecl_cc_ctx {
     int batch = 1;                        // batched two-hop gathers (R16, R19)
     int filter = 2;                       // R21 membership filter: 0 off, 1 on, 2 auto
     int order = 0;                        // 0 thread, warp, block; 1 block, warp, thread
+    int prejump = 2;                      // R23 pointer-doubling passes: 0 off, 1 on, 2 auto
     int *fa = nullptr, *fb = nullptr;     // spanning-forest outputs of the current call
     // CSR builder scratch (ecl_cc_build_csr; device, grow-only)
     void *csr_tmp = nullptr;

@@ -16,7 +16,7 @@ import paper_conf_hpdc_jaiganeshb18_b200 as ecl
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"thresh_thread": 16, "thresh_warp": 352, "load_mode": 1, "ttas": 1, "init": 3,
-            "jump": 4, "fini": 3, "batch": 1, "filter": 2}
+            "jump": 4, "fini": 3, "batch": 1, "filter": 2, "order": 0, "prejump": 2}
 
 
 @pytest.fixture(scope="module")
@@ -378,3 +378,29 @@ def test_forest_variants(h, opts):
 def test_forest_int64_offsets(h):
     g = gg.make_config("C5", seed=4, scale_down=9, device="cuda")
     assert_forest(h, g, index_dtype=torch.int64)
+
+
+# ---------------------------------------------------------------------------------------
+# R23 pointer-doubling passes between init and the hook kernels: forced on, forced off,
+# auto (default) — same labels; the grid configs (deep Init3 forests) trigger auto mode
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("prejump", [0, 1])
+def test_prejump_configs(h, name, prejump):
+    g = gg.make_config(name, seed=21, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, prejump=prejump)
+
+
+@pytest.mark.parametrize("g", hand_graphs(), ids=lambda g: g.name)
+def test_prejump_hand_built(h, g):
+    assert_parity(h, g, prejump=1)
+
+
+@pytest.mark.parametrize("prejump", [1, 2])
+def test_prejump_long_chains(h, prejump):
+    n = 1 << 20
+    v = torch.arange(1, n, dtype=torch.int64)
+    assert assert_parity(h, gg.csr_from_pairs("chain", n, v, v - 1), prejump=prejump) == 1
+    g = gg.make_config("C2", seed=3, scale_down=2, device="cuda")
+    assert_parity(h, g, prejump=prejump, filter=1)
+    assert_parity(h, g, prejump=prejump, jump=2, init=2)
