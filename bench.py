@@ -3,7 +3,8 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
 
-One "step" = one full ECL-CC run (init_bin, hook_thread, hook_warp, hook_block, finalize)
+One "step" = one full ECL-CC run (init_bin, depth_probe + prejump, hook_thread, hook_warp,
+hook_block, finalize)
 over the resident CSR of the workload (BASELINE.json configs; default C5 = Graph500
 Kronecker scale 27, edge factor 16, the config the metric's 1/2/4/8-GPU figure is quoted
 on).  For N > 1 (torchrun, one rank per GPU over NCCL) a step is the row-partitioned run
@@ -429,7 +430,9 @@ def main():
                          "L2 flushed (256 MB write) between timed steps",
                    "parallelism": f"rows{world}" if world > 1 else "single",
                    "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info},
-        "gpu_launches": 5 * args.steps if world == 1 else None,
+        # per run: init_bin, depth_probe, prejump (R23; exits at once on shallow forests),
+        # hook_thread, hook_range x2, finalize
+        "gpu_launches": 7 * args.steps if world == 1 else None,
         "clocks": clk.summary(),
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},
