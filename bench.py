@@ -410,7 +410,8 @@ def main():
                 "traffic": ncu_traffic(args.config, dom), "peak_source": peak_src,
                 "alg_bytes_per_launch": int(alg[dom]), "ms_per_launch": round(phase[dom], 4),
                 "path_alg_bytes": int(b_alg),
-                "path_frac": round(b_alg / (ms_step * 1e-3) / 1e9 / peak, 4)}
+                "path_frac": round(b_alg / (ms_step * 1e-3) / 1e9 / peak, 4),
+                "l2_probe_ceiling": l2_probe_ceiling(info, dom, phase[dom])}
     cpu = None
     cpu_paper = None
     if world == 1 and not args.no_cpu:
@@ -446,6 +447,26 @@ def main():
     if world > 1:
         tdist.barrier()
         tdist.destroy_process_group()
+
+
+def l2_probe_ceiling(info, kernel, ms):
+    """The binding resource of the hook kernels is L2 requests, one per probed edge
+    (DESIGN.md §5).  Compare the kernel with the measured ceiling of exactly that access
+    pattern (tools/l2_ceiling.py: stream the adjacency, probe one bitmap word for every
+    other entry, nothing else; profiles/l2_ceiling.json)."""
+    key = {"hook_block": "block_entries", "hook_warp": "warp_entries",
+           "hook_thread": "thread_entries"}.get(kernel)
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "l2_ceiling.json")))
+        rate = float(d["probe_pattern_entries_G_s"]) * 1e9
+    except Exception:
+        return None
+    if key is None or not info.get(key):
+        return None
+    t_ceil = info[key] / rate * 1e3
+    return {"entries": int(info[key]), "ceiling_entries_G_s": rate / 1e9,
+            "ms_at_ceiling": round(t_ceil, 4), "frac": round(t_ceil / ms, 4),
+            "source": "profiles/l2_ceiling.json (tools/l2_ceiling.py probe pattern)"}
 
 
 def ncu_traffic(config, kernel):
