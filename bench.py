@@ -314,12 +314,15 @@ def main():
     if world == 1:
         step = lambda: h.run(g.nindex, g.nlist, out=labels)  # noqa: E731
     else:
-        bounds = edist.partition_rows(g.nindex, world)
+        # rows split by estimated work (probed entries + a streaming share), outside the
+        # timed region like the graph itself
+        bounds = edist.partition_rows(g.nindex, world,
+                                      weights=edist.row_weights(g.nindex, g.nlist))
         lo, hi = bounds[rank], bounds[rank + 1]
         idx_r, lst_r = edist.slice_rows(g.nindex, g.nlist, lo, hi)
 
         def step():
-            parent = h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels)
+            parent = h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels, flatten=False)
             edist.forest_merge(parent, h, chunks=4)
 
     # ---- timed region ----

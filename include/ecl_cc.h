@@ -159,11 +159,14 @@ ECL_CC_API const char *ecl_cc_io_last_error(void);
  *   parent       n entries out (device): flattened min-ID labels of the subgraph formed by
  *                the edges stored in these rows (every vertex outside them labels itself
  *                unless joined through an edge).  Each undirected edge (a,b), a > b, is
- *                hooked by the owner of row a only (Fig. 6 line 1 "if (v > u)").
+ *                hooked by the owner of row a only (Fig. 6 line 1 "if (v > u)").  With
+ *                ECL_CC_OPT_STOP_AFTER = 2 the forest is left unflattened: parent[v] <= v
+ *                is some vertex of v's tree, enough to be a peer of ecl_cc_merge.
  * ecl_cc_merge: hook the edges (v, peer_labels[v - v_lo]) for v in [v_lo, v_hi) into the
- *   forest `parent` (every v whose peer label differs from v; peer_labels is a flattened
- *   min-ID labelling so peer_labels[v] <= v).  Does NOT flatten; call ecl_cc_finalize
- *   once after the last merge chunk.
+ *   forest `parent` (every v whose peer entry differs from v).  peer_labels is any forest
+ *   of the peer's subgraph with peer_labels[v] <= v in v's peer tree: a flattened min-ID
+ *   labelling or an unflattened parent array (the pairs (v, peer[v]) span the same trees,
+ *   P:L161-L163).  Does NOT flatten; call ecl_cc_finalize once after the last merge.
  * ecl_cc_finalize: parent[v] = root(v) for all v (Fini3). */
 ECL_CC_API ecl_cc_status ecl_cc_run_rows(ecl_cc_handle h, int32_t n, int32_t row_lo, int32_t row_hi,
                               int64_t m_rows, const int64_t *nindex_rows,

@@ -264,7 +264,11 @@ class Handle:
 
     # -- multi-GPU building blocks ----------------------------------------------------
     def run_rows(self, n: int, row_lo: int, row_hi: int, nindex_rows: torch.Tensor,
-                 nlist_rows: torch.Tensor, parent: Optional[torch.Tensor] = None, stream=None):
+                 nlist_rows: torch.Tensor, parent: Optional[torch.Tensor] = None, stream=None,
+                 flatten: bool = True):
+        """Local forest of rows [row_lo, row_hi) (ecl_cc_run_rows).  flatten=False leaves
+        the forest unflattened (ECL_CC_OPT_STOP_AFTER = 2): enough for ecl_cc_merge on a
+        peer, which saves one finalize per merge round."""
         d = self.device
         _dev_tensor(nindex_rows, "nindex_rows", (torch.int64,), d)
         _dev_tensor(nlist_rows, "nlist_rows", (torch.int32,), d)
@@ -273,10 +277,16 @@ class Handle:
         if parent is None:
             parent = torch.empty(n, dtype=torch.int32, device=d)
         _dev_tensor(parent, "parent", (torch.int32,), d)
-        self._check(self._lib.ecl_cc_run_rows(self._h, n, row_lo, row_hi, nlist_rows.numel(),
-                                              _ptr(nindex_rows),
-                                              _ptr(nlist_rows), _ptr(parent),
-                                              _stream_ptr(stream, d)))
+        if not flatten:
+            self.set_option("stop_after", 2)
+        try:
+            self._check(self._lib.ecl_cc_run_rows(self._h, n, row_lo, row_hi,
+                                                  nlist_rows.numel(), _ptr(nindex_rows),
+                                                  _ptr(nlist_rows), _ptr(parent),
+                                                  _stream_ptr(stream, d)))
+        finally:
+            if not flatten:
+                self.set_option("stop_after", 0)
         return parent
 
     def merge(self, parent: torch.Tensor, peer: torch.Tensor, v_lo: int = 0, stream=None):

@@ -5,8 +5,12 @@ rank owns a contiguous row range of the CSR chosen so every rank holds ~m/G entr
 builds a local forest of the edges stored in its rows with ``ecl_cc_run_rows`` (each
 undirected edge (a,b), a > b, is hooked only by the owner of row a: Fig. 6 line 1), then
 the forests are combined along a binomial tree: in round r the rank g with
-g mod 2^(r+1) == 2^r sends its flattened labels to g - 2^r, which receives them in chunks
-and hooks every (v, peer[v]) with ``ecl_cc_merge`` while the next chunk is in flight.
+g mod 2^(r+1) == 2^r sends its parent array to g - 2^r, which receives it in chunks and
+hooks every (v, peer[v]) with ``ecl_cc_merge`` while the next chunk is in flight; only
+rank 0's final forest is flattened (``ecl_cc_finalize``).  Rows are partitioned by
+estimated work (``row_weights``: probed entries u < v plus a streaming share of all
+entries), since the owner of high-ID rows probes most of its entries and the owner of
+low-ID rows almost none.
 Hook-once sufficiency makes the union of the forests' equivalence relations
 exact, so rank 0 ends with the same min-ID labels as a single-GPU run.
 
@@ -21,10 +25,42 @@ import torch
 import torch.distributed as dist
 
 
-def partition_rows(nindex: torch.Tensor, world: int) -> List[int]:
-    """Row bounds [b_0=0, ..., b_G=n] with ~m/G directed entries per range."""
+# Relative cost of an entry that is only streamed (u > v: Fig. 6 line 1 fails) against one
+# that is also probed/hooked (u < v), from the measured probe-pattern ceiling
+# (profiles/l2_ceiling.json: 2^30 entries streamed in ~0.66 ms, 2^29 probes ~1.38 ms more).
+STREAM_WEIGHT = 0.25
+
+
+def row_weights(nindex: torch.Tensor, nlist: torch.Tensor, chunk: int = 1 << 27) -> torch.Tensor:
+    """Per-row work estimate for partitioning: entries with u < v (each probed and maybe
+    hooked by the row's owner) + STREAM_WEIGHT x all entries (each streamed).  One pass
+    over nlist on its device (setup, outside any timed region).  Returns int64 weights
+    scaled by 4 (exact integers)."""
+    nindex = nindex.to(torch.int64)
+    n = nindex.numel() - 1
+    m = int(nindex[-1])
+    dev = nlist.device
+    nidx = nindex.to(dev)
+    lower = torch.zeros(n, dtype=torch.int64, device=dev)
+    for a in range(0, m, chunk):
+        pos = torch.arange(a, min(m, a + chunk), device=dev, dtype=torch.int64)
+        rows = torch.searchsorted(nidx, pos, right=True) - 1
+        lt = nlist[a:a + chunk].to(torch.int64) < rows
+        lower.index_add_(0, rows[lt], torch.ones(int(lt.sum()), dtype=torch.int64, device=dev))
+        del pos, rows, lt
+    deg = nidx[1:] - nidx[:-1]
+    return (4 * lower + int(4 * STREAM_WEIGHT) * deg).cpu()
+
+
+def partition_rows(nindex: torch.Tensor, world: int,
+                   weights: Optional[torch.Tensor] = None) -> List[int]:
+    """Row bounds [b_0=0, ..., b_G=n] with ~1/G of the total weight per range: by default
+    the directed entries (~m/G each), or per-row ``weights`` (e.g. ``row_weights``)."""
     nindex = nindex.to(torch.int64).cpu()
     n = nindex.numel() - 1
+    if weights is not None:
+        w = weights.to(torch.int64).cpu()
+        nindex = torch.cat([torch.zeros(1, dtype=torch.int64), torch.cumsum(w, 0)])
     m = int(nindex[-1])
     targets = torch.tensor([(m * g) // world for g in range(1, world)], dtype=torch.int64)
     cuts = torch.searchsorted(nindex, targets, right=False).clamp_(0, n).tolist()
@@ -81,7 +117,11 @@ def forest_merge(parent: torch.Tensor, ops, group=None, chunks: int = 4,
             for c in range(chunks):
                 works[c].wait()  # orders the compute stream after chunk c only
                 ops.merge(parent, peer[bounds[c]:bounds[c + 1]], bounds[c])
-            ops.finalize(parent)
+    # Only rank 0's final forest is flattened: a forest that is sent on or merged again
+    # needs no flattening, since (v, parent[v]) for every v spans the same trees as
+    # (v, root(v)) (hook-once sufficiency).
+    if rank == 0:
+        ops.finalize(parent)
     if broadcast:
         dist.broadcast(parent, src=_g(group, 0), group=group)
         return parent
@@ -104,5 +144,5 @@ def run_distributed(nindex: torch.Tensor, nlist: torch.Tensor, handle, group=Non
         bounds = partition_rows(nindex, world)
     lo, hi = bounds[rank], bounds[rank + 1]
     idx, lst = slice_rows(nindex, nlist, lo, hi)
-    parent = handle.run_rows(n, lo, hi, idx, lst)
+    parent = handle.run_rows(n, lo, hi, idx, lst, flatten=False)
     return forest_merge(parent, handle, group=group, chunks=chunks, broadcast=broadcast)

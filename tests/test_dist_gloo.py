@@ -33,6 +33,24 @@ def test_partition_rows_balanced_and_complete():
         assert max(per) - g.m / world <= dmax + 1
 
 
+def test_row_weights_count_probed_entries():
+    """row_weights = 4 x #{u < v in row v} + 1 x deg(v) (STREAM_WEIGHT = 1/4), checked
+    against a plain loop; the weighted partition balances those weights."""
+    g = gg.rmat(10, 8, seed=5)
+    nidx, nl = g.numpy()
+    w = edist.row_weights(g.nindex, g.nlist, chunk=1000).numpy()
+    for v in range(g.n):
+        row = nl[nidx[v]:nidx[v + 1]]
+        assert w[v] == 4 * int((row < v).sum()) + len(row)
+    tw = torch.from_numpy(w)
+    for world in (2, 3, 4, 8):
+        b = edist.partition_rows(g.nindex, world, weights=tw)
+        assert b[0] == 0 and b[-1] == g.n and all(b[i] <= b[i + 1] for i in range(world))
+        per = [int(tw[b[i]:b[i + 1]].sum()) for i in range(world)]
+        assert sum(per) == int(tw.sum())
+        assert max(per) - int(tw.sum()) / world <= int(tw.max()) + 1
+
+
 def test_tree_schedule_reaches_rank0():
     for world in range(1, 17):
         sched = edist.tree_schedule(world)

@@ -274,6 +274,29 @@ def test_fake_multi_gpu_merge(h, G):
     assert np.array_equal(acc.cpu().numpy(), expect)
 
 
+@pytest.mark.parametrize("G", [2, 3, 8])
+@pytest.mark.parametrize("name", ["C2", "C4", "C5"])
+def test_fake_multi_gpu_unflattened_tree_merge(h, name, G):
+    """dist.forest_merge's schedule on one GPU: work-weighted partition, unflattened local
+    forests (flatten=False), binomial-tree merges, one flatten at the end."""
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config(name, seed=4, scale_down=SMALL[name] + 1, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64, G, weights=dist.row_weights(nindex64, g.nlist))
+    forests = []
+    for r in range(G):
+        idx, lst = dist.slice_rows(nindex64, g.nlist, bounds[r], bounds[r + 1])
+        forests.append(h.run_rows(g.n, bounds[r], bounds[r + 1], idx, lst, flatten=False))
+    for (_, send, recv) in dist.tree_schedule(G):
+        chunks = [(c * g.n) // 3 for c in range(4)]
+        for c in range(3):
+            h.merge(forests[recv], forests[send][chunks[c]:chunks[c + 1]], chunks[c])
+    h.finalize(forests[0])
+    torch.cuda.synchronize()
+    assert np.array_equal(forests[0].cpu().numpy(), expect)
+
+
 # ---------------------------------------------------------------------------------------
 # paper ablations (SURVEY f1): every Init/Jump/Fini variant must give the same labels
 # ---------------------------------------------------------------------------------------
