@@ -33,7 +33,18 @@ __global__ void __launch_bounds__(256) random_kernel(long long P, const unsigned
     if (acc == 0x9e3779b9u) out[0] = acc;
 }
 
-template <int U>
+template <int F>
+__device__ __forceinline__ unsigned ld_probe(const unsigned *p)
+{
+    unsigned v;
+    if (F == 0) asm volatile("ld.global.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    else if (F == 1) asm volatile("ld.global.cg.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    else if (F == 2) asm volatile("ld.global.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    else asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+
+template <int U, int F = 0>
 __global__ void __launch_bounds__(256) probe_kernel(long long E, const int *list,
                                                     const unsigned *table, unsigned *out)
 {
@@ -51,8 +62,7 @@ __global__ void __launch_bounds__(256) probe_kernel(long long E, const int *list
 #pragma unroll
         for (int j = 0; j < U; j++) {
             w[j] = 0;
-            if ((u[j] & 1) == 0)
-                asm volatile("ld.global.b32 %0, [%1];" : "=r"(w[j]) : "l"(table + (u[j] >> 5)));
+            if ((u[j] & 1) == 0) w[j] = ld_probe<F>(table + (u[j] >> 5));
         }
 #pragma unroll
         for (int j = 0; j < U; j++) acc += w[j];
@@ -71,5 +81,18 @@ extern "C" int l2c_probe(long long E, const int *list, const unsigned *table, un
                          int grid)
 {
     probe_kernel<8><<<grid, 256>>>(E, list, table, out);
+    return (int)cudaGetLastError();
+}
+
+// probe-load flavour / loads-per-thread sweep: flavour 0 ld.global, 1 .cg, 2 L1::no_allocate,
+// 3 ld.relaxed.gpu; U = 4, 8 or 16 entries per thread per iteration
+extern "C" int l2c_probe_v(long long E, const int *list, const unsigned *table, unsigned *out,
+                           int grid, int flavour, int U)
+{
+#define L2C_CASE(UU, FF) if (U == UU && flavour == FF) probe_kernel<UU, FF><<<grid, 256>>>(E, list, table, out);
+    L2C_CASE(4, 0) L2C_CASE(4, 1) L2C_CASE(4, 2) L2C_CASE(4, 3)
+    L2C_CASE(8, 0) L2C_CASE(8, 1) L2C_CASE(8, 2) L2C_CASE(8, 3)
+    L2C_CASE(16, 0) L2C_CASE(16, 1) L2C_CASE(16, 2) L2C_CASE(16, 3)
+#undef L2C_CASE
     return (int)cudaGetLastError();
 }

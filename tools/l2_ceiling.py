@@ -63,6 +63,14 @@ def main():
     res["probe_pattern_ms_per_2^30_entries"] = round(ms, 3)
     res["probe_pattern_entries_G_s"] = round(E / ms / 1e6, 1)
     res["probe_pattern_sectors_G_s"] = round((E / 2 + E * 4 / 32) / ms / 1e6, 1)
+    if "--sweep" in sys.argv:
+        for U in (4, 8, 16):
+            for fl, nm in ((0, "ca"), (1, "cg"), (2, "noalloc"), (3, "relaxed_gpu")):
+                for gm in (4, 8):
+                    ms = timed(lambda: lib.l2c_probe_v(ctypes.c_longlong(E), ctypes.c_void_p(lst.data_ptr()),
+                                                       ctypes.c_void_p(table.data_ptr()),
+                                                       ctypes.c_void_p(out.data_ptr()), sms * gm, fl, U))
+                    res[f"probe_U{U}_{nm}_grid{gm}_entries_G_s"] = round(E / ms / 1e6, 1)
     print(json.dumps(res))
 
 
