@@ -22,6 +22,10 @@ namespace {
 constexpr int kCnt = 32;        // 64-bit counter words owned by the handle
 constexpr int kStatsOff = 16;   // ECL_CC_STATS counters live at cnt[16..31]
 constexpr int kNumStats = 16;
+#ifndef ECL_FAST_FINI
+#define ECL_FAST_FINI 1
+#endif
+constexpr bool kFastFini = ECL_FAST_FINI != 0;   // Fini3 via finalize3_kernel
 
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
 
@@ -187,8 +191,13 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             mark(4);
         }
         if (h->stop_after != 2) {
-            auto k = finalize_kernel<MODE>;
-            k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
+            if (h->fini == 3 && kFastFini) {
+                auto k = finalize3_kernel<MODE>;
+                k<<<grid_for(h, (const void *)k, ((long long)n + kFinPer - 1) / kFinPer), kBlock, 0, s>>>(n, parent);
+            } else {
+                auto k = finalize_kernel<MODE>;
+                k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
+            }
         }
         mark(5);
         if (tm && h->stop_after == 0) h->ev_valid = 1 + h->order;
@@ -351,8 +360,13 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
     if (!parent) return fail_arg(h, "null parent");
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
-    auto k = finalize_kernel<0>;
-    k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
+    if (h->fini == 3 && kFastFini) {
+        auto k = finalize3_kernel<0>;
+        k<<<grid_for(h, (const void *)k, ((long long)n + kFinPer - 1) / kFinPer), kBlock, 0, s>>>(n, parent);
+    } else {
+        auto k = finalize_kernel<0>;
+        k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
+    }
     CK(cudaGetLastError(), "finalize launch");
     return ECL_CC_OK;
 }
