@@ -335,14 +335,14 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
     const int cnt = v_hi - v_lo;
     if (h->load_mode == 1) {
         auto k = merge_hook_kernel<1>;
-        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
+        k<<<grid_for(h, (const void *)k, ((long long)cnt + 3) / 4), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
                                                                  , h->cnt + kStatsOff
 #endif
         );
     } else {
         auto k = merge_hook_kernel<0>;
-        k<<<grid_for(h, (const void *)k, cnt), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
+        k<<<grid_for(h, (const void *)k, ((long long)cnt + 3) / 4), kBlock, 0, s>>>(v_lo, cnt, peer_labels, parent, h->ttas
 #ifdef ECL_CC_STATS
                                                                  , h->cnt + kStatsOff
 #endif
