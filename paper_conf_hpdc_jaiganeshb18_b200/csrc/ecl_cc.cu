@@ -62,11 +62,15 @@ ecl_cc_status ensure_scratch(ecl_cc_handle h, int need, cudaStream_t s)
     if (need <= h->cap) return ECL_CC_OK;
     if (h->wl) CK(cudaFreeAsync(h->wl, s), "cudaFreeAsync(wl)");
     if (h->ub) CK(cudaFreeAsync(h->ub, s), "cudaFreeAsync(ub)");
+    if (h->tbits) CK(cudaFreeAsync(h->tbits, s), "cudaFreeAsync(tbits)");
     h->wl = nullptr;
     h->ub = nullptr;
+    h->tbits = nullptr;
     h->cap = 0;
     CK(cudaMallocAsync((void **)&h->wl, sizeof(int) * (size_t)need, s), "cudaMallocAsync(wl)");
     CK(cudaMallocAsync((void **)&h->ub, sizeof(unsigned) * (size_t)need, s), "cudaMallocAsync(ub)");
+    CK(cudaMallocAsync((void **)&h->tbits, sizeof(unsigned) * (((size_t)need + 31) / 32), s),
+       "cudaMallocAsync(tbits)");
     h->cap = need;
     return ECL_CC_OK;
 }
@@ -91,6 +95,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.parent = parent;
     p.wl = h->wl;
     p.ub = h->ub;
+    p.tbits = h->tbits;
     p.cap = h->cap;
     p.cnt = h->cnt;
     p.stats = h->cnt + kStatsOff;
@@ -266,6 +271,7 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
         cudaDeviceSynchronize();
         if (h->wl) cudaFree(h->wl);
         if (h->ub) cudaFree(h->ub);
+        if (h->tbits) cudaFree(h->tbits);
         if (h->cnt) cudaFree(h->cnt);
         if (h->flags) cudaFree(h->flags);
         if (h->e2e_index) cudaFree(h->e2e_index);

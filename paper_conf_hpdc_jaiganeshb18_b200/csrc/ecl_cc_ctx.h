@@ -15,6 +15,7 @@ struct ecl_cc_ctx {
     // scratch (device, grow-only)
     int *wl = nullptr;
     unsigned *ub = nullptr;
+    unsigned *tbits = nullptr;            // R24 thread-bin work bitmap (one bit per row)
     int cap = 0;
     unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [8..9] int
                                           // scheduling counters, [10] R21 anchor,
