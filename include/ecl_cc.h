@@ -199,7 +199,8 @@ typedef enum {
                                      128) for the device; 0 = leave unchanged.  NOTE: a
                                      device-wide setting that outlives the handle.       */
     ECL_CC_OPT_OCC_THREAD = 9,    /* blocks per SM of hook_thread (0 = max occupancy)     */
-    ECL_CC_OPT_OCC_RANGE = 10,    /* blocks per SM of hook_warp / hook_block (0 = max)    */
+    ECL_CC_OPT_OCC_RANGE = 10,    /* blocks per SM of hook_warp / hook_block (0 = max);
+                                     with ORDER 2: of hook_block only (0 = 3/4 of max)  */
     /* paper ablations; defaults are ECL-CC's */
     ECL_CC_OPT_INIT = 11,         /* 3 = Init3 first smaller neighbour (default),
                                      2 = Init2 smallest neighbour, 1 = Init1 own ID      */
@@ -211,9 +212,14 @@ typedef enum {
     ECL_CC_OPT_FILTER = 15,       /* anchor-tree membership bitmap (R21): 0 off,
                                      1 on, 2 (default) = on when 4n > 128 MB             */
     ECL_CC_OPT_ORDER = 16,        /* order of the three independent hook kernels: 0 =
-                                     thread, warp, block (paper, default); 1 =
-                                     block, warp, thread (hubs first).  Labels are the
-                                     same either way (R13).                            */
+                                     thread, warp, block (paper); 1 = block,
+                                     warp, thread (hubs first); 2 (default) = block on a
+                                     handle-owned side stream (forked from and joined
+                                     back into the run's stream with events) capped at
+                                     OCC_RANGE blocks/SM (0 = 3/4 of the SM), thread
+                                     then warp on the run's stream with full grids that
+                                     take the SM slots hook_block leaves or retires.
+                                     Labels are the same in every order (R13).         */
     ECL_CC_OPT_PREJUMP = 17       /* pointer-doubling passes between init and the hook
                                      kernels (R23; Jump's pointer jumping,
                                      P:L245, as synchronous passes): 0 off, 1 always,
@@ -244,7 +250,9 @@ ECL_CC_API ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int 
 
 /* Per-phase device time of the most recent full run with ECL_CC_OPT_TIMING set
  * (synchronises on it): ms[0] init_bin (incl. the counter memset), ms[1] hook_thread,
- * ms[2] hook_warp (worklist front), ms[3] hook_block (worklist back), ms[4] finalize. */
+ * ms[2] hook_warp (worklist front), ms[3] hook_block (worklist back), ms[4] finalize.
+ * With ECL_CC_OPT_ORDER 2 each hook kernel's span is measured on its own stream; the
+ * spans overlap, so ms[1] + ms[2] + ms[3] exceeds the hook phase of the run. */
 ECL_CC_API ecl_cc_status ecl_cc_get_timing(ecl_cc_handle h, float ms[5]);
 
 /* 1 if this build counts statistics (ECL_CC_STATS), else 0. */

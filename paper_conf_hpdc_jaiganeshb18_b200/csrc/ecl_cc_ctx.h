@@ -35,7 +35,10 @@ struct ecl_cc_ctx {
     int init_mode = 3, jump = 4, fini = 3; // paper ablation variants (defaults = ECL-CC)
     int batch = 1;                        // batched two-hop gathers (R16, R19)
     int filter = 2;                       // R21 membership filter: 0 off, 1 on, 2 auto
-    int order = 0;                        // 0 thread, warp, block; 1 block, warp, thread
+    int order = 2;                        // 0 thread, warp, block; 1 block, warp, thread;
+                                          // 2 (default) block on a side stream || thread, warp
+    cudaStream_t side = nullptr;          // order 2: hook_block's stream (lazy)
+    cudaEvent_t fork = nullptr, join = nullptr;
     int prejump = 2;                      // R23 pointer-doubling passes: 0 off, 1 on, 2 auto
     int *fa = nullptr, *fb = nullptr;     // spanning-forest outputs of the current call
     // CSR builder scratch (ecl_cc_build_csr; device, grow-only)
@@ -47,7 +50,7 @@ struct ecl_cc_ctx {
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks
     int timing = 0;                       // record per-kernel CUDA events
-    cudaEvent_t ev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev[8] = {};               // phase ends on the run's stream; [6..7] side stream
     int ev_valid = 0;
     // last run (for ecl_cc_get_worklist)
     cudaStream_t last_stream = nullptr;

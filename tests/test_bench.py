@@ -59,3 +59,13 @@ def test_l2_probe_ceiling_uses_the_committed_measurement():
     r = bench.l2_probe_ceiling({"block_entries": 526_200_000}, "hook_block", 2.0)
     assert r is not None and abs(r["ms_at_ceiling"] - 1.0) < 1e-3 and abs(r["frac"] - 0.5) < 1e-3
     assert bench.l2_probe_ceiling({}, "finalize", 1.0) is None
+
+
+def test_l2_probe_ceiling_of_the_concurrent_hook_group():
+    # order 2 runs the three hook kernels concurrently: the ceiling covers their entries
+    info = {"thread_entries": 100_000_000, "warp_entries": 200_000_000,
+            "block_entries": 226_200_000}
+    r = bench.l2_probe_ceiling(info, ("hook_thread", "hook_warp", "hook_block"), 2.0)
+    assert r["entries"] == 526_200_000
+    assert abs(r["ms_at_ceiling"] - 1.0) < 1e-3 and abs(r["frac"] - 0.5) < 1e-3
+    assert bench.l2_probe_ceiling(info, ("hook_block", "finalize"), 1.0) is None

@@ -16,7 +16,7 @@ import paper_conf_hpdc_jaiganeshb18_b200 as ecl
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"thresh_thread": 16, "thresh_warp": 352, "load_mode": 1, "ttas": 1, "init": 3,
-            "jump": 4, "fini": 3, "batch": 1, "filter": 2, "order": 0, "prejump": 2}
+            "jump": 4, "fini": 3, "batch": 1, "filter": 2, "order": 2, "prejump": 2}
 
 
 @pytest.fixture(scope="module")
@@ -350,6 +350,19 @@ def test_order_hubs_first(h, name):
     g = gg.make_config(name, seed=12, scale_down=SMALL[name], device="cuda")
     assert_parity(h, g, order=1)
     assert_parity(h, g, order=1, filter=1)
+    assert_parity(h, g, order=0)                  # the paper's order
+    assert_parity(h, g, order=0, filter=1)
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+def test_order_concurrent(h, name):
+    # hook_block on a side stream next to hook_warp + hook_thread (order 2): the three
+    # kernels hook the same edge sets concurrently; Fig. 6 is order-free (R13)
+    g = gg.make_config(name, seed=13, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, order=2)
+    assert_parity(h, g, order=2, filter=1)
+    assert_parity(h, g, order=2, filter=1, occ_range=2, occ_thread=6)
+    assert_parity(h, g, order=2, filter=1, occ_range=8)
 
 
 # ---------------------------------------------------------------------------------------

@@ -35,7 +35,7 @@ def main():
     ap.add_argument("--init", type=int, default=3)
     ap.add_argument("--fini", type=int, default=3)
     ap.add_argument("--occ-range", type=int, default=0)
-    ap.add_argument("--order", type=int, default=0)
+    ap.add_argument("--order", type=int, default=2)
     ap.add_argument("--prejump", type=int, default=2)
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=args.seed, device="cuda", scale_down=args.scale_down)
@@ -52,9 +52,14 @@ def main():
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
     res = []
     for _ in range(args.reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
         h.run(g.nindex, g.nlist, out=out)
+        e1.record()
         t = h.timing()
-        t["total"] = sum(t.values())
+        # the run's own span: with order 2 the hook kernels overlap (phases sum to more)
+        e1.synchronize()
+        t["total"] = e0.elapsed_time(e1)
         res.append(t)
     best = min(res, key=lambda r: r["total"])
     line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "order": args.order, "prejump": args.prejump, "n": g.n, "m": g.m, "mode": args.mode,
