@@ -78,7 +78,12 @@ ECL_CC_API ecl_cc_status ecl_cc_destroy(ecl_cc_handle h);
  *   nlist      m neighbour IDs (device)
  *   nstat_out  n labels out (device); also used as the union-find parent array during
  *              the run, so it must not alias nindex/nlist.
- * On completion nstat_out[v] = min{ w : w reachable from v }. */
+ * On completion nstat_out[v] = min{ w : w reachable from v }.
+ * Asynchrony: only enqueues work on `stream` (no host sync, no D2H); with the default
+ * kernel order (ECL_CC_OPT_ORDER 2) hook_block runs on a handle-owned side stream forked
+ * from and joined back into `stream` with events.  After one warm-up call has grown the
+ * handle's scratch for this graph size, a call can be captured into a CUDA graph and
+ * replayed (tests/test_gpu_parity.py::test_cuda_graph_capture_replay). */
 ECL_CC_API ecl_cc_status ecl_cc_run(ecl_cc_handle h, int32_t n, int64_t m, const int32_t *nindex,
                          const int32_t *nlist, int32_t *nstat_out, void *stream);
 

@@ -440,3 +440,32 @@ def test_prejump_long_chains(h, prejump):
     g = gg.make_config("C2", seed=3, scale_down=2, device="cuda")
     assert_parity(h, g, prejump=prejump, filter=1)
     assert_parity(h, g, prejump=prejump, jump=2, init=2)
+
+
+# ---------------------------------------------------------------------------------------
+# CUDA graph capture: ecl_cc_run only enqueues work on the caller's stream (the order-2
+# side stream is forked from and joined back into it with events), so a whole run can be
+# captured once and replayed; replays must give the oracle's labels every time
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("name,order", [("C4", 2), ("C4", 0), ("C2", 2), ("C5", 2)])
+def test_cuda_graph_capture_replay(h, name, order):
+    g = gg.make_config(name, seed=21, scale_down=SMALL[name], device="cuda")
+    nidx, nl = g.numpy()
+    expect, _ = oracle.bfs(nidx, nl)
+    h.set_option("order", order)     # C2 also captures R23's cooperative pass kernel
+    try:
+        out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            h.run(g.nindex, g.nlist, out=out)     # warm-up: grows the handle's scratch
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=s):
+            h.run(g.nindex, g.nlist, out=out)
+        for _ in range(3):
+            out.fill_(-1)
+            graph.replay()
+            torch.cuda.synchronize()
+            assert np.array_equal(out.cpu().numpy(), expect)
+    finally:
+        h.set_option("order", DEFAULTS["order"])
