@@ -11,7 +11,7 @@ transfer + merge/chunks.  Projected step = max over ranks of the local forest + 
 of rounds + rank 0's finalize.  The merged labels are checked against the single-GPU
 labels.  --even uses the plain m/G entry split instead of the work-weighted one.
 
-    python tools/mgpu_emulate.py [--config C5] [--gpus 1,2,4,8] [--link-gbs 750]
+    python tools/mgpu_emulate.py [--config C5] [--gpus 1,2,4,8] [--link-gbs 750] [--order 2]
 """
 import argparse
 import json
@@ -46,10 +46,12 @@ def main():
     ap.add_argument("--link-gbs", type=float, default=750.0)
     ap.add_argument("--chunks", type=int, default=4)
     ap.add_argument("--even", action="store_true")
+    ap.add_argument("--order", type=int, default=2, help="ECL_CC_OPT_ORDER of every run")
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=1, device="cuda")
     n, m = g.n, g.m
     h = ecl.Handle(0)
+    h.set_option("order", args.order)
     nidx64 = g.nindex.to(torch.int64)
     ref = torch.empty(n, dtype=torch.int32, device="cuda")
     t1, _ = timed(lambda: h.run(g.nindex, g.nlist, out=ref))
