@@ -213,6 +213,9 @@ def test_argument_errors(h):
     assert lib.ecl_cc_run(h._h, -1, 0, None, None, None, None) == 1
     assert lib.ecl_cc_run(h._h, 4, 2**31, idx.data_ptr(), None, None, None) == 1
     assert lib.ecl_cc_run(h._h, 0, 0, None, None, None, None) == 0
+    for bad in (-1, 3):                       # kernel orders are 0, 1, 2
+        with pytest.raises(ecl.EclCCError, match="order"):
+            h.set_option("order", bad)
 
 
 def test_validate(h):
