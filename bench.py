@@ -124,34 +124,51 @@ def build_graph(name: str, seed: int, device, scale_down: int = 0):
 
 
 def algorithmic_bytes(g, parent_init, hw):
-    """Per-phase algorithmic (compulsory, streamed) bytes of one run.
-    parent_init = Init3 parents (stop_after=1 run) on the device."""
+    """Per-kernel split of B_alg = S_idx(n+1) + 4m + 4n: every
+    byte of B_alg is charged to exactly ONE kernel, so the parts sum to B_alg.
+      init_bin     nindex (S_idx per offset) + the entries of every row no hook kernel
+                   reads (Init3 roots — init scans their whole row, R3 — and the
+                   thread-bin rows of <= 4 entries whose smaller entries all equal the
+                   Init parent, R24 — init holds their whole row in registers)
+      hook_thread  4 B per entry of the active thread-bin rows with hook work (R24)
+      hook_warp    4 B per entry of the worklist-front rows (17..352)
+      hook_block   4 B per entry of the worklist-back rows (> 352)
+      finalize     4 B per label written
+    parent_init = Init3 parents (a stop_after=1 run) on the device."""
     n, m = g.n, g.m
     s_idx = g.nindex.element_size()
     deg = g.degrees()
-    v = torch.arange(n, device=g.nindex.device, dtype=torch.int64)
-    active = parent_init.to(torch.int64) != v
-    # Init3 reads row entries up to the first smaller one (rows are sorted by the
-    # generators, so that is 1 entry when one exists, else the whole row)
-    first = g.nlist[g.nindex[:-1].to(torch.int64).clamp(max=max(m - 1, 0))].to(torch.int64)
-    scanned = torch.where(deg == 0, torch.zeros_like(deg),
-                          torch.where(first < v, torch.ones_like(deg), deg))
+    dev = g.nindex.device
+    v = torch.arange(n, device=dev, dtype=torch.int64)
+    par = parent_init.to(torch.int64)
+    active = par != v
     t1, t2 = hw
     thr = active & (deg <= t1)
     fr = active & (deg > t1) & (deg <= t2)
     bk = active & (deg > t2)
-    e_thr, e_fr, e_bk = (int(deg[x].sum()) for x in (thr, fr, bk))
-    n_fr, n_bk = int(fr.sum()), int(bk.sum())
+    # R24: a thread-bin row of <= 4 entries needs hook work only if it has a smaller entry
+    # other than its Init parent (rows of 5..16 entries are all treated as work)
+    small = thr & (deg <= 4)
+    other = torch.zeros(n, dtype=torch.bool, device=dev)
+    starts = g.nindex[:-1].to(torch.int64)
+    for j in range(4):
+        sel = small & (deg > j)
+        x = g.nlist[starts[sel] + j].to(torch.int64)
+        other[sel] = other[sel] | ((x < v[sel]) & (x != par[sel]))
+    tw = thr & (~small | other)
+    e_thr, e_fr, e_bk = (int(deg[x].sum()) for x in (tw, fr, bk))
     b = {
-        "init_bin": s_idx * (n + 1) + 4 * n + 4 * int(scanned.sum()) + 8 * (n_fr + n_bk),
-        "hook_thread": s_idx * (n + 1) + 4 * n + 4 * e_thr,
-        "hook_warp": 8 * n_fr + 2 * s_idx * n_fr + 4 * e_fr,
-        "hook_block": 8 * n_bk + 2 * s_idx * n_bk + 4 * e_bk,
-        "finalize": 8 * n,
+        "init_bin": s_idx * (n + 1) + 4 * (m - e_thr - e_fr - e_bk),
+        "hook_thread": 4 * e_thr,
+        "hook_warp": 4 * e_fr,
+        "hook_block": 4 * e_bk,
+        "finalize": 4 * n,
     }
-    info = {"active": int(active.sum()), "thread_vertices": int(thr.sum()), "thread_entries": e_thr,
-            "warp_vertices": n_fr, "warp_entries": e_fr, "block_vertices": n_bk,
-            "block_entries": e_bk, "hooked_entries": None}
+    assert sum(b.values()) == s_idx * (n + 1) + 4 * m + 4 * n
+    info = {"active": int(active.sum()), "thread_bin_vertices": int(thr.sum()),
+            "thread_vertices": int(tw.sum()), "thread_entries": e_thr,
+            "warp_vertices": int(fr.sum()), "warp_entries": e_fr,
+            "block_vertices": int(bk.sum()), "block_entries": e_bk}
     return b, info
 
 
@@ -180,30 +197,59 @@ def time_steps(fn, K, W, stream, flush_buf=None):
     return per
 
 
-def cpu_oracle_sample(config: str, seed: int, budget_s: float = 15.0):
-    """Time the oracle (O1 BFS, 1 thread) on a bounded sample of the same workload: the
-    same generator recipe scaled down until one run fits the budget."""
-    import oracle
-    sd = {"C1": 0, "C2": 0, "C3": 0, "C4": 1, "C5": 3}[config]
+# One bounded sample of every workload, used by BOTH oracle timings (cpu_baseline on
+# rank 0 of our arm, and the reference arm): the same generator recipe with 2^-sd of the
+# vertices (C5: 1/8 -> n = 2^24, m ~ 0.52e9; one O1 run ~3 s on one core).
+SAMPLE_SD = {"C1": 0, "C2": 0, "C3": 0, "C4": 1, "C5": 3}
+
+
+class PinnedCore:
+    """Run the oracle pinned to one host core (`taskset -c 0`): the first
+    core this process may use; the affinity is restored afterwards."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = min(self.prev)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.prev)
+
+
+def oracle_sample(config: str, seed: int):
+    sd = SAMPLE_SD[config]
     g, _ = build_graph(config, seed, "cuda" if torch.cuda.is_available() else "cpu", sd)
     nidx, nl = g.numpy()
     del g
+    return sd, nidx, nl
+
+
+def sample_text(config, sd, nidx, nl, core):
+    return (f"{config} recipe at 1/2^{sd} scale (n={nidx.shape[0] - 1}, m={int(nl.shape[0])}), "
+            f"O1 serial BFS, pinned to host core {core} of {os.cpu_count()}")
+
+
+def cpu_oracle_sample(config: str, seed: int, budget_s: float = 15.0):
+    """Time the oracle (O1 BFS, 1 thread pinned to one core) on the bounded sample of the
+    workload (SAMPLE_SD), repeated up to 5 times within the budget."""
+    import oracle
+    sd, nidx, nl = oracle_sample(config, seed)
     oracle.build()
-    t0 = time.perf_counter()
-    _, ncc = oracle.bfs(nidx, nl)
-    dt = time.perf_counter() - t0
-    reps = 1
-    while dt * (reps + 1) / reps < budget_s and reps < 5:
-        t1 = time.perf_counter()
+    with PinnedCore() as pc:
+        t0 = time.perf_counter()
         oracle.bfs(nidx, nl)
-        dt += time.perf_counter() - t1
-        reps += 1
+        dt = time.perf_counter() - t0
+        reps = 1
+        while dt * (reps + 1) / reps < budget_s and reps < 5:
+            t1 = time.perf_counter()
+            oracle.bfs(nidx, nl)
+            dt += time.perf_counter() - t1
+            reps += 1
     m = int(nl.shape[0])
     out = {"value": round(m * reps / dt / 1e6, 3), "unit": "Medges/s", "cores": 1,
            "kind": "oracle",
-           "sample": f"{config} recipe at 1/2^{sd} scale (n={nidx.shape[0]-1}, m={m}), "
-                     f"O1 serial BFS, {reps} run(s), {dt:.2f} s, single thread of "
-                     f"{os.cpu_count()} host cores"}
+           "sample": sample_text(config, sd, nidx, nl, pc.core) + f", {reps} run(s), {dt:.2f} s"}
     return out, (nidx, nl)
 
 
@@ -232,23 +278,23 @@ def cpu_paper_codes(nidx, nl, budget_s: float = 10.0):
 
 
 def run_reference(args):
-    """Reference arm = the CPU oracle as it stands, on a bounded sample of the workload."""
+    """Reference arm = the CPU oracle as it stands (O1, one pinned core) on the bounded
+    sample of the workload (SAMPLE_SD, the same sample as our arm's cpu_baseline); under
+    torchrun only rank 0 runs and prints, the other ranks exit without work."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import oracle
-    sd = {"C1": 0, "C2": 1, "C3": 2, "C4": 4, "C5": 6}[args.config]
-    g, _ = build_graph(args.config, args.seed, "cuda" if torch.cuda.is_available() else "cpu", sd)
-    nidx, nl = g.numpy()
-    del g
+    sd, nidx, nl = oracle_sample(args.config, args.seed)
     oracle.build()
-    for _ in range(args.warmup):
-        oracle.bfs(nidx, nl)
-    per = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        oracle.bfs(nidx, nl)
-        per.append(time.perf_counter() - t0)
+    with PinnedCore() as pc:
+        for _ in range(args.warmup):
+            oracle.bfs(nidx, nl)
+        per = []
+        for _ in range(args.steps):
+            t0 = time.perf_counter()
+            oracle.bfs(nidx, nl)
+            per.append(time.perf_counter() - t0)
     m = int(nl.shape[0])
     tot = sum(per)
     value = m * args.steps / tot / 1e6
@@ -260,12 +306,53 @@ def run_reference(args):
         "config": {"workload": args.config, "description": CONFIG_TEXT[args.config],
                    "sample_scale_down": sd, "n": int(nidx.shape[0] - 1), "m": m},
         "cpu_baseline": {"value": round(value, 3), "unit": "Medges/s", "cores": 1,
-                         "kind": "oracle",
-                         "sample": f"{args.config} recipe at 1/2^{sd} scale, O1 serial BFS"},
+                         "kind": "oracle", "sample": sample_text(args.config, sd, nidx, nl,
+                                                                 pc.core)},
         "e2e": {"value": round(value, 3), "unit": "Medges/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
+
+
+def relaunch_with_torchrun(n: int) -> int:
+    """`bench.py --gpus N` without a torchrun environment: launch the N ranks ourselves
+    (one process per GPU, the driver's own launch line) and return their exit code."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={n}", "--master-addr=127.0.0.1", f"--master-port={port}",
+           os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
+def check_world(args) -> None:
+    """Run here only if the world matches --gpus: without a torchrun environment and
+    N > 1, launch the N ranks ourselves (and exit with their code), or fail loudly when
+    the node has fewer than N GPUs; under torchrun, WORLD_SIZE must equal N."""
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print(f"bench.py: --gpus {args.gpus} needs {args.gpus} GPUs, this node has {have}",
+                  file=sys.stderr)
+            sys.exit(2)
+        sys.exit(relaunch_with_torchrun(args.gpus))
+    _, world, _ = dist_env()
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        sys.exit(2)
+
+
+def launches_per_step(world: int, rank: int, chunks: int) -> int:
+    """Our kernels per step: init_bin, depth_probe, prejump (exits at once on shallow
+    forests), hook_thread, hook_range x2, finalize; with G ranks: + identity_outside, one
+    merge_hook per received chunk, and finalize on rank 0 only."""
+    if world == 1:
+        return 7
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
+    recv = sum(1 for (_, _s, r) in edist.tree_schedule(world) if r == rank)
+    return 7 + recv * chunks + (1 if rank == 0 else 0)
 
 
 def main():
@@ -278,12 +365,14 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--load-mode", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--chunks", type=int, default=4, help="merge chunks per round (N > 1)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--check", action="store_true", help="full oracle parity of the bench run")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    check_world(args)
 
     rank, world, local = dist_env()
     torch.cuda.set_device(local)
@@ -297,33 +386,41 @@ def main():
     g, gen_s = build_graph(args.config, args.seed, dev)
     n, m = g.n, g.m
     s_idx = g.nindex.element_size()
+    idx_dtype = str(g.nindex.dtype).replace("torch.", "")
     h = ecl.Handle(local)
     h.set_option("load_mode", args.load_mode)
     stream = torch.cuda.current_stream(dev)
     labels = torch.empty(n, dtype=torch.int32, device=dev)
     flush_buf = None if (m * 4 > 2 * L2_BYTES) else torch.zeros(64 * 2 ** 20, dtype=torch.int32,
                                                                   device=dev)
-
-    # ---- algorithmic-bytes bookkeeping (outside the timed region) ----
-    h.set_option("stop_after", 1)
-    h.run(g.nindex, g.nlist, out=labels)
-    h.set_option("stop_after", 0)
-    alg, info = algorithmic_bytes(g, labels, (16, 352))
     b_alg = s_idx * (n + 1) + 4 * m + 4 * n
+
+    # ---- algorithmic-bytes bookkeeping (outside the timed region; N=1 path) ----
+    alg, info = {}, {}
+    if world == 1:
+        h.set_option("stop_after", 1)
+        h.run(g.nindex, g.nlist, out=labels)
+        h.set_option("stop_after", 0)
+        alg, info = algorithmic_bytes(g, labels, (16, 352))
 
     if world == 1:
         step = lambda: h.run(g.nindex, g.nlist, out=labels)  # noqa: E731
     else:
-        # rows split by estimated work (probed entries + a streaming share), outside the
-        # timed region like the graph itself
+        # rows split by estimated work (probed entries + a streaming share); every rank
+        # keeps ONLY its slice resident (the full graph is built once to cut it, outside
+        # the timed region, and released)
         bounds = edist.partition_rows(g.nindex, world,
                                       weights=edist.row_weights(g.nindex, g.nlist))
         lo, hi = bounds[rank], bounds[rank + 1]
         idx_r, lst_r = edist.slice_rows(g.nindex, g.nlist, lo, hi)
+        idx_r, lst_r = idx_r.clone(), lst_r.clone()
+        del g
+        torch.cuda.empty_cache()
+        slice_entries = int(lst_r.numel())
 
         def step():
             parent = h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels, flatten=False)
-            edist.forest_merge(parent, h, chunks=4)
+            edist.forest_merge(parent, h, chunks=args.chunks)
 
     # ---- timed region ----
     if world > 1:
@@ -374,45 +471,66 @@ def main():
         h.set_option("timing", 0)
         hooks_ms = run_ms - phase["init_bin"] - phase["finalize"]
 
-    # ---- parity of the bench output (invariants on the device; full oracle with --check) --
+    # ---- parity of the bench output: I1/I2 invariants on the device ----
+    # (with N ranks the labels are broadcast and every rank checks I1 on its own slice)
     ok = None
-    if rank == 0:
-        lab = labels.to(torch.int64)
-        i1 = True
-        nidx64 = g.nindex.to(torch.int64)
-        chunk = 1 << 28
-        for a in range(0, m, chunk):
-            pos = torch.arange(a, min(m, a + chunk), device=dev, dtype=torch.int64)
-            rows = torch.searchsorted(nidx64, pos, right=True) - 1
-            i1 &= bool((lab[rows] == lab[g.nlist[a:a + chunk].to(torch.int64)]).all())
-            del pos, rows
-        del nidx64
-        ar = torch.arange(n, device=dev)
-        i2 = bool((lab <= ar).all()) and bool((lab[lab] == lab).all())
-        ok = {"I1": i1, "I2": i2, "components": int((lab == ar).sum())}
-        del lab, ar
+    if world == 1:
+        ok = device_invariants(g.nindex, g.nlist, labels, 0, dev)
         if args.check:
             import oracle
             exp, ncc = oracle.bfs(*g.numpy())
             ok["oracle_exact"] = bool(np.array_equal(labels.cpu().numpy(), exp))
+    else:
+        tdist.broadcast(labels, src=0)
+        mine = device_invariants(idx_r, lst_r, labels, lo, dev)
+        flag = torch.tensor([int(mine["I1"]), int(mine["I2"])], dtype=torch.int32, device=dev)
+        tdist.all_reduce(flag, op=tdist.ReduceOp.MIN)
+        ok = {"I1": bool(flag[0]), "I2": bool(flag[1]), "components": mine["components"]}
 
     # ---- end-to-end through the public API with host buffers ----
     e2e = None
-    if not args.no_e2e and world == 1:
-        hidx = g.nindex.cpu().pin_memory()
-        hlst = g.nlist.cpu().pin_memory()
-        hout = torch.empty(n, dtype=torch.int32).pin_memory()
-        h.run_host(hidx, hlst, out=hout)
-        ts = []
-        for _ in range(args.e2e_steps):
-            t0 = time.perf_counter()
+    if not args.no_e2e:
+        if world == 1:
+            hidx = g.nindex.cpu().pin_memory()
+            hlst = g.nlist.cpu().pin_memory()
+            hout = torch.empty(n, dtype=torch.int32).pin_memory()
             h.run_host(hidx, hlst, out=hout)
-            ts.append(time.perf_counter() - t0)
-        e2e = {"value": round(m / (sum(ts) / len(ts)) / 1e6, 3), "unit": "Medges/s",
-               "h2d_bytes_per_step": int(hidx.numel() * hidx.element_size() + hlst.numel() * 4),
-               "d2h_bytes_per_step": int(n * 4), "steps": len(ts),
-               "ms_per_step": round(1e3 * sum(ts) / len(ts), 3)}
-        del hidx, hlst, hout
+            ts = []
+            for _ in range(args.e2e_steps):
+                t0 = time.perf_counter()
+                h.run_host(hidx, hlst, out=hout)
+                ts.append(time.perf_counter() - t0)
+            e2e_ms = 1e3 * sum(ts) / len(ts)
+            h2d = int(hidx.numel() * hidx.element_size() + hlst.numel() * 4)
+            del hidx, hlst, hout
+        else:
+            # every rank copies its slice host->device, runs its rows, merges; rank 0
+            # copies the labels back (device-timed per rank, max over ranks)
+            hidx = idx_r.cpu().pin_memory()
+            hlst = lst_r.cpu().pin_memory()
+            hout = torch.empty(n, dtype=torch.int32).pin_memory()
+            didx, dlst = torch.empty_like(idx_r), torch.empty_like(lst_r)
+
+            def e2e_step():
+                didx.copy_(hidx, non_blocking=True)
+                dlst.copy_(hlst, non_blocking=True)
+                parent = h.run_rows(n, lo, hi, didx, dlst, parent=labels, flatten=False)
+                edist.forest_merge(parent, h, chunks=args.chunks)
+                if rank == 0:
+                    hout.copy_(labels, non_blocking=True)
+
+            pe = time_steps(e2e_step, args.e2e_steps, 1, stream)
+            t = torch.tensor([sum(pe) / len(pe)], dtype=torch.float64, device=dev)
+            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+            hb = torch.tensor([hidx.numel() * 8 + hlst.numel() * 4], dtype=torch.int64,
+                              device=dev)
+            tdist.all_reduce(hb)
+            h2d = int(hb.item())
+            del hidx, hlst, hout, didx, dlst
+        e2e = {"value": round(m / (e2e_ms * 1e-3) / 1e6, 3), "unit": "Medges/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": int(n * 4),
+               "steps": args.e2e_steps, "ms_per_step": round(e2e_ms, 3)}
 
     if rank != 0:
         if world > 1:
@@ -424,10 +542,12 @@ def main():
     roof = None
     if phase:
         # the three hook kernels run concurrently (order 2), so the dominant unit is the
-        # concurrent hook group: its algorithmic bytes over the span from init's end to
-        # the join (run span minus init and finalize); per-kernel spans overlap
+        # concurrent hook group: the bytes of B_alg charged to them (algorithmic_bytes: the
+        # entries of the rows they stream) over the span from init's end to the join (run
+        # span minus init and finalize); per-kernel spans overlap
         hk = ("hook_thread", "hook_warp", "hook_block")
         alg_h = sum(alg[k] for k in hk)
+        assert alg_h <= b_alg
         achieved = alg_h / (hooks_ms * 1e-3) / 1e9
         tr = [ncu_traffic(args.config, k) for k in hk]
         roof = {"bound": "hbm", "kernel": "hook_thread+hook_warp||hook_block (concurrent)",
@@ -437,6 +557,7 @@ def main():
                 "alg_bytes_per_launch": int(alg_h), "ms_per_launch": round(hooks_ms, 4),
                 "path_alg_bytes": int(b_alg),
                 "path_frac": round(b_alg / (ms_step * 1e-3) / 1e9 / peak, 4),
+                "alg_bytes_by_kernel": alg,
                 "l2_probe_ceiling": l2_probe_ceiling(info, hk, hooks_ms)}
         dom = max(phase_seq, key=phase_seq.get)
         a_seq = alg[dom] / (phase_seq[dom] * 1e-3) / 1e9
@@ -445,6 +566,14 @@ def main():
             "achieved": round(a_seq, 1), "frac": round(a_seq / peak, 4),
             "traffic": ncu_traffic(args.config, dom),
             "l2_probe_ceiling": l2_probe_ceiling(info, (dom,), phase_seq[dom])}
+    elif world > 1:
+        # whole-job roofline: B_alg over the max-over-ranks step time and N x peak (SURVEY
+        # §8(d) multi-GPU figure)
+        roof = {"bound": "hbm", "kernel": "whole step (run_rows + forest merge)",
+                "achieved": round(b_alg / (ms_step * 1e-3) / 1e9, 1), "peak": peak * world,
+                "unit": "GB/s", "frac": round(b_alg / (ms_step * 1e-3) / 1e9 / (peak * world), 4),
+                "traffic": None, "peak_source": peak_src + f" x {world} GPUs",
+                "path_alg_bytes": int(b_alg)}
     cpu = None
     cpu_paper = None
     if world == 1 and not args.no_cpu:
@@ -458,15 +587,14 @@ def main():
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "int32", "data": "synthetic",
         "config": {"workload": args.config, "description": CONFIG_TEXT[args.config],
-                   "seed": args.seed, "n": n, "m": m,
-                   "index_dtype": str(g.nindex.dtype).replace("torch.", ""),
+                   "seed": args.seed, "n": n, "m": m, "index_dtype": idx_dtype,
                    "l2": "inputs larger than L2" if flush_buf is None else
                          "L2 flushed (256 MB write) between timed steps",
                    "parallelism": f"rows{world}" if world > 1 else "single",
-                   "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info},
-        # per run: init_bin, depth_probe, prejump (R23; exits at once on shallow forests),
-        # hook_thread, hook_range x2, finalize
-        "gpu_launches": 7 * args.steps if world == 1 else None,
+                   "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info,
+                   **({"rank0_rows": [lo, hi], "rank0_entries": slice_entries,
+                       "merge_chunks": args.chunks} if world > 1 else {})},
+        "gpu_launches": launches_per_step(world, rank, args.chunks) * args.steps,
         "clocks": clk.summary(),
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},
@@ -481,6 +609,23 @@ def main():
     if world > 1:
         tdist.barrier()
         tdist.destroy_process_group()
+
+
+def device_invariants(nindex, nlist, labels, row_lo, dev, chunk=1 << 28):
+    """I1 (both endpoints of every entry of rows [row_lo, row_lo + len(nindex) - 1) share a
+    label) and I2 (label[v] <= v, labels are fixed points) on the device."""
+    lab = labels.to(torch.int64)
+    nidx64 = nindex.to(torch.int64)
+    m = int(nlist.numel())
+    i1 = True
+    for a in range(0, m, chunk):
+        pos = torch.arange(a, min(m, a + chunk), device=dev, dtype=torch.int64)
+        rows = torch.searchsorted(nidx64, pos, right=True) - 1 + row_lo
+        i1 &= bool((lab[rows] == lab[nlist[a:a + chunk].to(torch.int64)]).all())
+        del pos, rows
+    ar = torch.arange(lab.numel(), device=dev)
+    i2 = bool((lab <= ar).all()) and bool((lab[lab] == lab).all())
+    return {"I1": i1, "I2": i2, "components": int((lab == ar).sum())}
 
 
 def l2_probe_ceiling(info, kernel, ms):

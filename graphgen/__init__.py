@@ -296,6 +296,47 @@ def make_config(name: str, seed: int = 1, device="cpu", scale_down: int = 0) -> 
     raise KeyError(name)
 
 
+def raw_csr(name: str, n: int, rows: torch.Tensor, cols: torch.Tensor,
+            seed: Optional[int] = None, index_dtype: Optional[torch.dtype] = None) -> Graph:
+    """CSR of the directed entries (rows[i], cols[i]) exactly as given — no symmetrising,
+    no loop removal, no dedupe — with every row's entries in a seeded random order, or in
+    their given order when ``seed`` is None."""
+    rows = rows.to(torch.int64)
+    cols = cols.to(torch.int64)
+    device = rows.device
+    E = rows.numel()
+    i = torch.arange(E, dtype=torch.int64, device=device)
+    key = (rows << 32) | (i if seed is None else hi32(hash64(seed, 4343, i)))
+    order = torch.argsort(key)
+    nlist = cols[order].to(torch.int32).contiguous()
+    nindex = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    if E:
+        torch.cumsum(torch.bincount(rows, minlength=n), 0, out=nindex[1:])
+    if index_dtype is None:
+        index_dtype = torch.int32 if E < 2 ** 31 else torch.int64
+    return Graph(name, n, nindex.to(index_dtype), nlist)
+
+
+def inject_loops_dups(g: Graph, seed: int, p_loop: float = 0.1, p_dup: float = 0.1) -> Graph:
+    """A raw CSR with the same components as ``g`` (whose entries are kept): a self-loop
+    (v, v) added to each vertex with probability p_loop, each directed entry (a, b)
+    duplicated with probability p_dup together with a copy of (b, a) (so the input stays
+    symmetric), and every row's entries shuffled, so loops and duplicates land anywhere in
+    a row (also among the first entries Init3 reads).  SURVEY §8(b) "accepted inputs"."""
+    device = g.nlist.device
+    deg = g.degrees()
+    rows = torch.repeat_interleave(torch.arange(g.n, dtype=torch.int64, device=device), deg)
+    cols = g.nlist.to(torch.int64)
+    v = torch.arange(g.n, dtype=torch.int64, device=device)
+    loop = v[hi32(hash64(seed, 4444, v)) < int(p_loop * (1 << 32))]
+    e = torch.arange(g.m, dtype=torch.int64, device=device)
+    dup = e[hi32(hash64(seed, 4545, e)) < int(p_dup * (1 << 32))]
+    R = torch.cat([rows, loop, rows[dup], cols[dup]])
+    C = torch.cat([cols, loop, cols[dup], rows[dup]])
+    return raw_csr(g.name + f"_loopdup{seed}", g.n, R, C, seed,
+                   index_dtype=g.nindex.dtype)
+
+
 def shuffle_rows(g: Graph, seed: int) -> Graph:
     """Randomly permute the entries inside every row (reading R4: order-independence)."""
     deg = g.degrees()

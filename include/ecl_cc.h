@@ -36,7 +36,9 @@
  *     error text is available from ecl_cc_last_error(h).  n == 0 is a no-op returning OK.
  *   - A handle may be used by one host thread at a time.  It owns device scratch (the
  *     double-sided worklist and counters, O(n)), allocated stream-ordered on first use,
- *     grown on demand, and released by ecl_cc_destroy.
+ *     grown on demand, and released by ecl_cc_destroy.  Calls on one handle are ordered:
+ *     a call enqueued on a stream other than the previous call's first makes its stream
+ *     wait (cudaStreamWaitEvent) for the previous call, since they share the scratch.
  */
 #ifndef ECL_CC_H
 #define ECL_CC_H
@@ -67,8 +69,9 @@ typedef enum {
  * allocations).  *out is set to NULL on failure. */
 ECL_CC_API ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device);
 
-/* Release the handle and its scratch.  NULL is a no-op.  Synchronises the handle's device
- * before freeing. */
+/* Release the handle and its scratch.  NULL is a no-op.  No device-wide synchronisation:
+ * the scratch is freed stream-ordered after the handle's most recent call, and the host
+ * waits only for that (the handle's own work), not for other work on the device. */
 ECL_CC_API ecl_cc_status ecl_cc_destroy(ecl_cc_handle h);
 
 /* Connected components of the whole graph (int32 offsets; requires m <= INT32_MAX).
@@ -203,7 +206,9 @@ typedef enum {
     ECL_CC_OPT_L2_FETCH = 8,      /* cudaLimitMaxL2FetchGranularity hint in bytes (32, 64,
                                      128) for the device; 0 = leave unchanged.  NOTE: a
                                      device-wide setting that outlives the handle.       */
-    ECL_CC_OPT_OCC_THREAD = 9,    /* blocks per SM of hook_thread (0 = max occupancy)     */
+    ECL_CC_OPT_OCC_THREAD = 9,    /* blocks per SM of hook_thread (0 = max occupancy);
+                                     with ORDER 2 it caps hook_warp as well (both run
+                                     on the caller's stream next to hook_block)         */
     ECL_CC_OPT_OCC_RANGE = 10,    /* blocks per SM of hook_warp / hook_block (0 = max);
                                      with ORDER 2: of hook_block only (0 = 3/4 of max)  */
     /* paper ablations; defaults are ECL-CC's */

@@ -83,7 +83,6 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     ecl_cc_status st = ensure_scratch(h, nrows > 0 ? nrows : 1, s);
     if (st != ECL_CC_OK) return st;
     CK(cudaMemsetAsync(h->cnt, 0, kCnt * sizeof(unsigned long long), s), "cudaMemsetAsync");
-    h->last_stream = s;
 
     Params p;
     p.n = n;
@@ -183,11 +182,6 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         if (h->order == 2) {
             // concurrent: hub chunks (L2-request bound) on a side stream next to the
             // warp and thread bins (issue / latency bound), occupancy split per SM
-            if (!h->side) {
-                CK(cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking), "side stream");
-                CK(cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming), "fork event");
-                CK(cudaEventCreateWithFlags(&h->join, cudaEventDisableTiming), "join event");
-            }
             const size_t sm = hook_smem_bytes<idx_t>();
             const int full = blocks_per_sm(
                 h, (const void *)hook_range_kernel<MODE, idx_t, kUnitFront, true>, sm);
@@ -197,6 +191,10 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             // (3/4 of the SM's blocks measured best at C5: 12.99 vs 13.48 ms sequential)
             const int cb = h->occ_range > 0 ? h->occ_range : std::max(1, (3 * full) / 4);
             const int cw = h->occ_thread;
+            // the side stream and both events exist for the handle's lifetime (created
+            // together in ecl_cc_create); once the fork is recorded the join is always
+            // recorded and waited on, so no error return leaves work of this call running
+            // on the side stream unordered with `stream`
             CK(cudaEventRecord(h->fork, s), "fork");
             CK(cudaStreamWaitEvent(h->side, h->fork, 0), "fork wait");
             if (tm) cudaEventRecord(h->ev[6], h->side);
@@ -216,8 +214,12 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
                 k<<<grid_for(h, (const void *)k, -1, sm, cw), kBlock, sm, s>>>(p);
             }
             mark(3);
-            CK(cudaEventRecord(h->join, h->side), "join");
-            CK(cudaStreamWaitEvent(s, h->join, 0), "join wait");
+            cudaError_t ej = cudaEventRecord(h->join, h->side);
+            if (ej == cudaSuccess) ej = cudaStreamWaitEvent(s, h->join, 0);
+            if (ej != cudaSuccess) {
+                cudaStreamSynchronize(h->side);   // cannot order it on `stream`: drain it
+                return fail_cuda(h, ej, "join");
+            }
             mark(4);
         } else if (h->order == 1) {
             block_k();
@@ -267,12 +269,16 @@ ecl_cc_status run_impl(ecl_cc_handle h, int32_t n, int64_t m, const idx_t *ninde
     DeviceGuard g(h->device);
     if (!g.ok) return fail_arg(h, "cannot select the handle's device");
     cudaStream_t s = (cudaStream_t)stream;
+    ecl_cc_status st = begin_call(h, s);
+    if (st != ECL_CC_OK) return st;
     switch (h->load_mode) {
-    case 0: return launch_path<0, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
-    case 2: return launch_path<2, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
-    case 3: return launch_path<3, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
-    default: return launch_path<1, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode);
+    case 0: st = launch_path<0, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode); break;
+    case 2: st = launch_path<2, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode); break;
+    case 3: st = launch_path<3, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode); break;
+    default: st = launch_path<1, idx_t>(h, n, m, row_lo, nrows, nindex, nlist, out, s, rows_mode); break;
     }
+    ecl_cc_status se = end_call(h, s);
+    return st != ECL_CC_OK ? st : se;
 }
 
 }  // namespace
@@ -290,11 +296,28 @@ ecl_cc_status ecl_cc_create(ecl_cc_handle *out, int device)
     if (!h) return ECL_CC_ERR_OOM;
     h->device = device;
     DeviceGuard g(device);
+    // everything the handle owns for its lifetime is created here, all or nothing: the
+    // side stream (hook_block under order 2; the stream destroy frees on), the fork/join
+    // events of the concurrent order, the end-of-call event, the counters
     cudaError_t e = cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-    if (e == cudaSuccess) e = cudaMalloc((void **)&h->cnt, kCnt * sizeof(unsigned long long));
-    if (e == cudaSuccess) e = cudaMalloc((void **)&h->flags, 4 * sizeof(int));
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->join, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->done, cudaEventDisableTiming);
+    if (e == cudaSuccess)
+        e = cudaMallocAsync((void **)&h->cnt, kCnt * sizeof(unsigned long long), h->side);
+    if (e == cudaSuccess) e = cudaMallocAsync((void **)&h->flags, 4 * sizeof(int), h->side);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->side);
     if (e != cudaSuccess) {
-        if (h->cnt) cudaFree(h->cnt);
+        if (h->side) {
+            if (h->cnt) cudaFreeAsync(h->cnt, h->side);
+            if (h->flags) cudaFreeAsync(h->flags, h->side);
+            cudaStreamSynchronize(h->side);
+            cudaStreamDestroy(h->side);
+        }
+        if (h->fork) cudaEventDestroy(h->fork);
+        if (h->join) cudaEventDestroy(h->join);
+        if (h->done) cudaEventDestroy(h->done);
         delete h;
         return e == cudaErrorMemoryAllocation ? ECL_CC_ERR_OOM : ECL_CC_ERR_CUDA;
     }
@@ -306,23 +329,23 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
 {
     if (!h) return ECL_CC_OK;
     {
+        // no device-wide synchronisation: the frees are stream-ordered on the handle's own
+        // stream after the handle's last call (its `done` event), and only that stream is
+        // waited for
         DeviceGuard g(h->device);
-        cudaDeviceSynchronize();
-        if (h->wl) cudaFree(h->wl);
-        if (h->ub) cudaFree(h->ub);
-        if (h->tbits) cudaFree(h->tbits);
-        if (h->cnt) cudaFree(h->cnt);
-        if (h->flags) cudaFree(h->flags);
-        if (h->e2e_index) cudaFree(h->e2e_index);
-        if (h->e2e_list) cudaFree(h->e2e_list);
-        if (h->e2e_labels) cudaFree(h->e2e_labels);
-        if (h->gbits) cudaFree(h->gbits);
-        if (h->csr_tmp) cudaFree(h->csr_tmp);
+        cudaStream_t s = h->side;
+        if (h->done_valid) cudaStreamWaitEvent(s, h->done, 0);
+        void *bufs[] = {h->wl, h->ub, h->tbits, h->cnt, h->flags, h->e2e_index, h->e2e_list,
+                        h->e2e_labels, h->gbits, h->csr_tmp};
+        for (void *b : bufs)
+            if (b) cudaFreeAsync(b, s);
+        cudaStreamSynchronize(s);
         for (int i = 0; i < 8; i++)
             if (h->ev[i]) cudaEventDestroy(h->ev[i]);
-        if (h->fork) cudaEventDestroy(h->fork);
-        if (h->join) cudaEventDestroy(h->join);
-        if (h->side) cudaStreamDestroy(h->side);
+        cudaEventDestroy(h->fork);
+        cudaEventDestroy(h->join);
+        cudaEventDestroy(h->done);
+        cudaStreamDestroy(s);
     }
     delete h;
     return ECL_CC_OK;
@@ -380,6 +403,8 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
     if (!peer_labels || !parent) return fail_arg(h, "null pointer");
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
+    ecl_cc_status st = begin_call(h, s);
+    if (st != ECL_CC_OK) return st;
     const int cnt = v_hi - v_lo;
     if (h->load_mode == 1) {
         auto k = merge_hook_kernel<1>;
@@ -397,7 +422,7 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
         );
     }
     CK(cudaGetLastError(), "merge_hook launch");
-    return ECL_CC_OK;
+    return end_call(h, s);
 }
 
 ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream)
@@ -408,6 +433,8 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
     if (!parent) return fail_arg(h, "null parent");
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
+    ecl_cc_status st = begin_call(h, s);
+    if (st != ECL_CC_OK) return st;
     if (h->fini == 3 && kFastFini) {
         auto k = finalize3_kernel<0>;
         k<<<grid_for(h, (const void *)k, ((long long)n + kFinPer - 1) / kFinPer), kBlock, 0, s>>>(n, parent);
@@ -416,7 +443,7 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
         k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, parent, h->fini);
     }
     CK(cudaGetLastError(), "finalize launch");
-    return ECL_CC_OK;
+    return end_call(h, s);
 }
 
 ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, const void *nindex_host,
@@ -431,6 +458,10 @@ ecl_cc_status ecl_cc_run_host(ecl_cc_handle h, int32_t n, int64_t m, const void 
     if (index_bytes == 4 && m > INT32_MAX) return fail_arg(h, "m > INT32_MAX with int32 offsets");
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
+    {
+        ecl_cc_status st = begin_call(h, s);
+        if (st != ECL_CC_OK) return st;
+    }
     const size_t ib = (size_t)index_bytes * ((size_t)n + 1);
     if (ib > h->e2e_index_bytes) {
         if (h->e2e_index) CK(cudaFreeAsync(h->e2e_index, s), "cudaFreeAsync");
@@ -476,6 +507,11 @@ ecl_cc_status ecl_cc_validate(ecl_cc_handle h, int32_t n, int64_t m, const void 
     if (!nindex || (m > 0 && !nlist)) return fail_arg(h, "null pointer");
     DeviceGuard g(h->device);
     cudaStream_t s = (cudaStream_t)stream;
+    {
+        ecl_cc_status st = begin_call(h, s);
+        if (st != ECL_CC_OK) return st;
+        h->last_stream = s;   // every return below follows a synchronisation of `s`
+    }
     int flags = 0;
     CK(cudaMemsetAsync(h->flags, 0, sizeof(int), s), "memset");
     const int grid = (int)std::min<long long>(((long long)n + kBlock) / kBlock, 148LL * 8);

@@ -107,6 +107,11 @@ ecl_cc_status ecl_cc_build_csr(ecl_cc_handle h, int32_t n, int64_t num_edges, co
     if (!g.ok) return fail_arg(h, "cannot select the handle's device");
     cudaStream_t s = (cudaStream_t)stream;
     *m_out = 0;
+    {
+        ecl_cc_status st = begin_call(h, s);
+        if (st != ECL_CC_OK) return st;
+        h->last_stream = s;   // every return below follows a synchronisation of `s`
+    }
     const int grid = h->sms * 8;
     if (num_edges == 0 || n == 0) {
         if (num_edges > 0) return fail_arg(h, "edges given for an empty vertex set");

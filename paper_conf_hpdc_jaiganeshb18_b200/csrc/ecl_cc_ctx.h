@@ -37,8 +37,11 @@ struct ecl_cc_ctx {
     int filter = 2;                       // R21 membership filter: 0 off, 1 on, 2 auto
     int order = 2;                        // 0 thread, warp, block; 1 block, warp, thread;
                                           // 2 (default) block on a side stream || thread, warp
-    cudaStream_t side = nullptr;          // order 2: hook_block's stream (lazy)
+    cudaStream_t side = nullptr;          // handle-owned stream: hook_block under order 2,
+                                          //   and the stream destroy() frees on
     cudaEvent_t fork = nullptr, join = nullptr;
+    cudaEvent_t done = nullptr;           // recorded at the end of every enqueueing call
+    bool done_valid = false;
     int prejump = 2;                      // R23 pointer-doubling passes: 0 off, 1 on, 2 auto
     int *fa = nullptr, *fb = nullptr;     // spanning-forest outputs of the current call
     // CSR builder scratch (ecl_cc_build_csr; device, grow-only)
@@ -78,6 +81,32 @@ inline ecl_cc_status fail_arg(ecl_cc_handle h, const char *msg)
         cudaError_t e_ = (call);                             \
         if (e_ != cudaSuccess) return fail_cuda(h, e_, where); \
     } while (0)
+
+// Stream ordering of the handle's scratch across calls.  begin_call: a call on a stream
+// other than the previous call's waits for that call (the scratch is shared), end_call:
+// record where this call ends.  Skipped while `s` is being captured into a CUDA graph
+// (the graph replays in the capturing stream's order).
+inline bool capturing(cudaStream_t s)
+{
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    return cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone;
+}
+
+inline ecl_cc_status begin_call(ecl_cc_handle h, cudaStream_t s)
+{
+    if (h->done_valid && h->last_stream != s && !capturing(s))
+        CK(cudaStreamWaitEvent(s, h->done, 0), "wait for the handle's previous call");
+    return ECL_CC_OK;
+}
+
+inline ecl_cc_status end_call(ecl_cc_handle h, cudaStream_t s)
+{
+    h->last_stream = s;
+    if (capturing(s)) return ECL_CC_OK;
+    CK(cudaEventRecord(h->done, s), "record call end");
+    h->done_valid = true;
+    return ECL_CC_OK;
+}
 
 // Make `dev` current for the duration of a call, restoring the caller's device.
 struct DeviceGuard {

@@ -95,35 +95,51 @@ def tree_schedule(world: int):
 
 def forest_merge(parent: torch.Tensor, ops, group=None, chunks: int = 4,
                  broadcast: bool = False) -> Optional[torch.Tensor]:
-    """Combine every rank's flattened forest ``parent`` (n labels) into rank 0's.
+    """Combine every rank's forest ``parent`` (n entries, flattened or not) into rank 0's.
 
     Returns the global labels on rank 0 (and on every rank if ``broadcast``), else None.
-    ``ops`` provides merge(parent, peer_chunk, v_lo) and finalize(parent)."""
+    ``ops`` provides merge(parent, peer_chunk, v_lo) and finalize(parent).  With NCCL the
+    device chunks go straight over NVLink; with gloo (CPU transport: the multi-process
+    tests) device chunks are staged through host memory."""
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
     n = parent.numel()
+    staged = parent.is_cuda and dist.get_backend(group) == "gloo"
     bounds = [(n * c) // chunks for c in range(chunks + 1)]
     peer = None
     for (_, send, recv) in tree_schedule(world):
         if rank == send:
             for c in range(chunks):
-                dist.send(parent[bounds[c]:bounds[c + 1]], dst=_g(group, recv), group=group)
+                part = parent[bounds[c]:bounds[c + 1]]
+                dist.send(part.cpu() if staged else part, dst=_g(group, recv), group=group)
             break
         if rank == recv:
             if peer is None:
                 peer = torch.empty_like(parent)
-            works = [dist.irecv(peer[bounds[c]:bounds[c + 1]], src=_g(group, send), group=group)
+                if staged:
+                    host = torch.empty(n, dtype=parent.dtype, pin_memory=True)
+            buf = host if staged else peer
+            works = [dist.irecv(buf[bounds[c]:bounds[c + 1]], src=_g(group, send), group=group)
                      for c in range(chunks)]
             for c in range(chunks):
                 works[c].wait()  # orders the compute stream after chunk c only
+                if staged:
+                    peer[bounds[c]:bounds[c + 1]].copy_(host[bounds[c]:bounds[c + 1]])
                 ops.merge(parent, peer[bounds[c]:bounds[c + 1]], bounds[c])
+            if staged:
+                torch.cuda.current_stream(parent.device).synchronize()  # host buffer reuse
     # Only rank 0's final forest is flattened: a forest that is sent on or merged again
     # needs no flattening, since (v, parent[v]) for every v spans the same trees as
     # (v, root(v)) (hook-once sufficiency, P:L161-L163).
     if rank == 0:
         ops.finalize(parent)
     if broadcast:
-        dist.broadcast(parent, src=_g(group, 0), group=group)
+        if staged:
+            host = parent.cpu()
+            dist.broadcast(host, src=_g(group, 0), group=group)
+            parent.copy_(host)
+        else:
+            dist.broadcast(parent, src=_g(group, 0), group=group)
         return parent
     return parent if rank == 0 else None
 

@@ -5,6 +5,7 @@ import os
 import subprocess
 import sys
 
+import numpy as np
 import torch
 
 import bench
@@ -38,21 +39,36 @@ def test_reference_arm_other_ranks_are_silent():
     assert not [ln for ln in out.splitlines() if ln.startswith("{")]
 
 
-def test_algorithmic_bytes_partition_the_rows():
-    """Per-bin entries add up to the entries of active rows, bins follow R2/R3."""
-    g = gg.make_config("C4", seed=3, scale_down=8)
-    nidx, nl = g.numpy()
-    init3 = torch.from_numpy(oracle.init3(nidx, nl))
-    alg, info = bench.algorithmic_bytes(g, init3, (16, 352))
-    deg = g.degrees()
-    active = init3.to(torch.int64) != torch.arange(g.n)
-    assert info["active"] == int(active.sum())
-    assert (info["thread_entries"] + info["warp_entries"] + info["block_entries"]
-            == int(deg[active].sum()))
-    assert info["thread_vertices"] == int((active & (deg <= 16)).sum())
-    assert info["block_vertices"] == int((active & (deg > 352)).sum())
-    assert alg["finalize"] == 8 * g.n
-    assert all(v >= 0 for v in alg.values())
+def test_algorithmic_bytes_partition_b_alg():
+    """The per-kernel parts sum to B_alg = S_idx(n+1) + 4m + 4n; bins follow
+    R2/R3 and the thread-bin work rows follow R24, checked against a plain loop."""
+    for name, sd in (("C4", 8), ("C1", 2), ("C2", 8)):
+        g = gg.shuffle_rows(gg.make_config(name, seed=3, scale_down=sd), seed=1)
+        nidx, nl = g.numpy()
+        init3 = oracle.init3(nidx, nl)
+        alg, info = bench.algorithmic_bytes(g, torch.from_numpy(init3), (16, 352))
+        s_idx = g.nindex.element_size()
+        assert sum(alg.values()) == s_idx * (g.n + 1) + 4 * g.m + 4 * g.n
+        assert alg["finalize"] == 4 * g.n and all(x >= 0 for x in alg.values())
+        e = {"thread": 0, "warp": 0, "block": 0}
+        nv = {"thread": 0, "warp": 0, "block": 0}
+        for v in range(g.n):
+            row = nl[nidx[v]:nidx[v + 1]]
+            p = init3[v]
+            if p == v:
+                continue
+            d = len(row)
+            if d <= 16:
+                if d <= 4 and not any(x < v and x != p for x in row):
+                    continue
+                k = "thread"
+            else:
+                k = "warp" if d <= 352 else "block"
+            e[k] += d
+            nv[k] += 1
+        for k in e:
+            assert info[f"{k}_entries"] == e[k] and info[f"{k}_vertices"] == nv[k], (name, k)
+        assert info["active"] == int((init3 != np.arange(g.n)).sum())
 
 
 def test_l2_probe_ceiling_uses_the_committed_measurement():
@@ -69,3 +85,23 @@ def test_l2_probe_ceiling_of_the_concurrent_hook_group():
     assert r["entries"] == 526_200_000
     assert abs(r["ms_at_ceiling"] - 1.0) < 1e-3 and abs(r["frac"] - 0.5) < 1e-3
     assert bench.l2_probe_ceiling(info, ("hook_block", "finalize"), 1.0) is None
+
+
+def test_gpus_flag_fails_without_enough_gpus():
+    """`bench.py --gpus 2` without a torchrun environment launches 2 ranks itself, and
+    fails loudly (no silent 1-rank line) on a node with fewer GPUs."""
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    env.pop("WORLD_SIZE", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2",
+                        "--steps", "1", "--config", "C1"], capture_output=True, text=True,
+                       env=env, timeout=300)
+    assert r.returncode != 0 and "needs 2 GPUs" in r.stderr
+    assert not [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+
+
+def test_gpus_flag_must_match_world():
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="", WORLD_SIZE="3", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2",
+                        "--steps", "1", "--config", "C1"], capture_output=True, text=True,
+                       env=env, timeout=300)
+    assert r.returncode != 0 and "WORLD_SIZE=3" in r.stderr

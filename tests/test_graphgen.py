@@ -67,3 +67,27 @@ def test_grid_deletion_rate():
     g = gg.grid2d(256, 256, 0.10, seed=1)
     full = 2 * 2 * 256 * 255
     assert abs(g.m / full - 0.9) < 0.01
+
+
+def test_inject_loops_dups_raw_csr():
+    """The raw-CSR generator keeps every original entry, adds loops and (symmetric)
+    duplicates, and leaves the components unchanged (oracle O1 on both)."""
+    import oracle
+    g = gg.make_config("C1", seed=2, scale_down=4)
+    r = gg.inject_loops_dups(g, seed=3, p_loop=0.2, p_dup=0.2)
+    ni, nl = r.numpy()
+    ni = ni.astype(np.int64)
+    assert ni[0] == 0 and ni[-1] == len(nl) and np.all(np.diff(ni) >= 0)
+    rows = np.repeat(np.arange(r.n), np.diff(ni))
+    assert np.any(rows == nl), "no self-loop injected"
+    key = rows.astype(np.int64) * r.n + nl
+    assert len(np.unique(key)) < len(key), "no duplicate injected"
+    assert np.any(np.diff(key) < 0), "rows not shuffled"
+    # same multiset of distinct non-loop entries as the clean graph, and symmetric
+    clean = np.unique(key[rows != nl])
+    g_ni, g_nl = g.numpy()
+    g_rows = np.repeat(np.arange(g.n), np.diff(g_ni.astype(np.int64)))
+    assert np.array_equal(clean, g_rows.astype(np.int64) * g.n + g_nl)
+    rkey = nl.astype(np.int64) * r.n + rows
+    assert np.array_equal(np.sort(rkey), np.sort(key))
+    assert np.array_equal(oracle.bfs(ni, nl)[0], oracle.bfs(*g.numpy())[0])

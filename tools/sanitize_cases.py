@@ -1,0 +1,93 @@
+"""Small cases for compute-sanitizer: memcheck / racecheck / synccheck.
+
+    compute-sanitizer --tool racecheck python tools/sanitize_cases.py [--quick]
+
+Runs the hand-built graphs (clean and raw: loops, duplicates, unsorted rows) and C1 / a
+scaled C2 / C4 / C5 through ecl_cc_run, ecl_cc_run_i64, the spanning forest and the
+multi-GPU building blocks (run_rows -> merge -> finalize), under kernel orders 0 and 2,
+with the R23 prejump passes forced on (cooperative grid barrier) and off, and the R21
+bitmap filter forced on; every result is compared with oracle O1.  Exit code 1 on any
+mismatch.
+"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+import oracle  # noqa: E402
+import paper_conf_hpdc_jaiganeshb18_b200 as ecl  # noqa: E402
+from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist  # noqa: E402
+
+
+def cases(quick):
+    from test_gpu_parity import hand_graphs
+    from test_gpu_raw_csr import hand_raw_graphs
+    G = [g for g in hand_graphs() if g.n <= 5000] + hand_raw_graphs()[:5]
+    G.append(gg.make_config("C1", seed=1))
+    G.append(gg.inject_loops_dups(gg.make_config("C1", seed=2, scale_down=2), seed=1))
+    if not quick:
+        G.append(gg.make_config("C2", seed=1, scale_down=10))
+        G.append(gg.make_config("C4", seed=1, scale_down=12))
+        G.append(gg.make_config("C5", seed=1, scale_down=14))
+    return G
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--quick", action="store_true")
+    args = ap.parse_args()
+    bad = 0
+    runs = 0
+    with ecl.Handle(0) as h:
+        for g in cases(args.quick):
+            gd = g.to("cuda")
+            expect, _ = oracle.bfs(*g.numpy())
+            for order in (0, 2):
+                for prejump in (0, 1):
+                    for filt in (0, 1):
+                        h.set_option("order", order).set_option("prejump", prejump)
+                        h.set_option("filter", filt)
+                        for idx in (gd.nindex, gd.nindex.to(torch.int64)):
+                            out = h.run(idx, gd.nlist)
+                            torch.cuda.synchronize()
+                            runs += 1
+                            if not np.array_equal(out.cpu().numpy(), expect):
+                                print(f"MISMATCH {g.name} order={order} prejump={prejump} "
+                                      f"filter={filt} idx={idx.dtype}", flush=True)
+                                bad += 1
+            h.set_option("order", 2).set_option("prejump", 1).set_option("filter", 2)
+            lab, ta, tb = h.spanning_forest(gd.nindex, gd.nlist)
+            torch.cuda.synchronize()
+            runs += 1
+            if not np.array_equal(lab.cpu().numpy(), expect) or oracle.check_forest(
+                    *g.numpy(), expect, ta.cpu().numpy(), tb.cpu().numpy()) != 0:
+                print(f"FOREST MISMATCH {g.name}", flush=True)
+                bad += 1
+            # multi-GPU building blocks: 3 fake ranks, tree merge, one flatten
+            nidx64 = gd.nindex.to(torch.int64)
+            b = edist.partition_rows(nidx64.cpu(), 3)
+            forests = []
+            for r in range(3):
+                i, l_ = edist.slice_rows(nidx64, gd.nlist, b[r], b[r + 1])
+                forests.append(h.run_rows(g.n, b[r], b[r + 1], i, l_, flatten=False))
+            for (_, s, rcv) in edist.tree_schedule(3):
+                h.merge(forests[rcv], forests[s])
+            h.finalize(forests[0])
+            torch.cuda.synchronize()
+            runs += 1
+            if not np.array_equal(forests[0].cpu().numpy(), expect):
+                print(f"MERGE MISMATCH {g.name}", flush=True)
+                bad += 1
+    print(f"sanitize_cases: {runs} runs, {bad} mismatches", flush=True)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
