@@ -344,12 +344,16 @@ def check_world(args) -> None:
         sys.exit(2)
 
 
-def launches_per_step(world: int, rank: int, chunks: int) -> int:
-    """Our kernels per step: init_bin, depth_probe, prejump (exits at once on shallow
-    forests), hook_thread, hook_range x2, finalize; with G ranks: + identity_outside, one
-    merge_hook per received chunk, and finalize on rank 0 only."""
+def launches_per_step(world: int, rank: int, chunks: int, merge: str) -> int:
+    """Our kernels per step on `rank`: init_bin, depth_probe, prejump (exits at once on
+    shallow forests), hook_thread, hook_range x2, finalize; with G ranks: identity_outside
+    instead of finalize in run_rows, then for the tree merge one merge_hook per received
+    chunk and rank 0's finalize, for the encoded merges finalize + encode on every rank
+    g > 0 and merge_bits + merge_pairs + finalize on rank 0."""
     if world == 1:
         return 7
+    if merge != "tree":
+        return 7 + (3 if rank == 0 else 2)
     from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
     recv = sum(1 for (_, _s, r) in edist.tree_schedule(world) if r == rank)
     return 7 + recv * chunks + (1 if rank == 0 else 0)
@@ -365,7 +369,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--load-mode", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--chunks", type=int, default=4, help="merge chunks per round (N > 1)")
+    ap.add_argument("--chunks", type=int, default=4, help="tree merge: chunks per round")
+    ap.add_argument("--merge", default="p2p", choices=["p2p", "compact", "tree"],
+                    help="N > 1: forest merge (dist.EncodedMerge p2p / compact, or the "
+                         "binomial tree of full forests)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--check", action="store_true", help="full oracle parity of the bench run")
@@ -417,12 +424,21 @@ def main():
         del g
         torch.cuda.empty_cache()
         slice_entries = int(lst_r.numel())
+        merger = None
+        if args.merge != "tree":
+            merger = edist.EncodedMerge(h, n, edist.row_anchor(idx_r, lo), mode=args.merge)
+
+        def merge(parent):
+            if merger is None:
+                edist.forest_merge(parent, h, chunks=args.chunks)
+            else:
+                merger(parent)
 
         def step():
-            parent = h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels, flatten=False)
-            edist.forest_merge(parent, h, chunks=args.chunks)
+            merge(h.run_rows(n, lo, hi, idx_r, lst_r, parent=labels, flatten=False))
 
     # ---- timed region ----
+    merger = merger if world > 1 else None
     if world > 1:
         tdist.barrier()
     torch.cuda.synchronize()
@@ -514,8 +530,7 @@ def main():
             def e2e_step():
                 didx.copy_(hidx, non_blocking=True)
                 dlst.copy_(hlst, non_blocking=True)
-                parent = h.run_rows(n, lo, hi, didx, dlst, parent=labels, flatten=False)
-                edist.forest_merge(parent, h, chunks=args.chunks)
+                merge(h.run_rows(n, lo, hi, didx, dlst, parent=labels, flatten=False))
                 if rank == 0:
                     hout.copy_(labels, non_blocking=True)
 
@@ -532,6 +547,10 @@ def main():
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": int(n * 4),
                "steps": args.e2e_steps, "ms_per_step": round(e2e_ms, 3)}
 
+    if world > 1 and merger is not None:
+        torch.cuda.synchronize()
+        tdist.barrier()
+        merger.close()
     if rank != 0:
         if world > 1:
             tdist.barrier()
@@ -593,8 +612,9 @@ def main():
                    "parallelism": f"rows{world}" if world > 1 else "single",
                    "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info,
                    **({"rank0_rows": [lo, hi], "rank0_entries": slice_entries,
-                       "merge_chunks": args.chunks} if world > 1 else {})},
-        "gpu_launches": launches_per_step(world, rank, args.chunks) * args.steps,
+                       "merge": args.merge, "merge_chunks": args.chunks}
+                      if world > 1 else {})},
+        "gpu_launches": launches_per_step(world, rank, args.chunks, args.merge) * args.steps,
         "clocks": clk.summary(),
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},

@@ -183,6 +183,46 @@ ECL_CC_API ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, 
                            const int32_t *peer_labels, int32_t *parent, void *stream);
 ECL_CC_API ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream);
 
+/* ---- encoded forest exchange and P2P merge (not in the paper) ----------
+ * ecl_cc_forest_encode: encode a FLATTENED labelling `labels` (n entries, labels[v] the
+ *   root of v's tree, e.g. the output of ecl_cc_run_rows without STOP_AFTER 2, or of
+ *   ecl_cc_finalize) as the relation it spans: D = labels[anchor] (pick a vertex of the
+ *   largest component, e.g. the highest-degree row), bits[v / 32] bit v % 32 set iff
+ *   labels[v] == D, and the pairs (v, labels[v]) of every other v with labels[v] != v.
+ *   The edges {(v, D) : bit v} u {(v, labels[v]) : pairs} span exactly the classes of
+ *   `labels`, so merging them is exact (hook-once sufficiency).
+ *     bits   (n + 31) / 32 uint32 words out (device)
+ *     pairs  2 x cap int32 out (device): pair i is (pairs[2i], pairs[2i+1]); the order is
+ *            unspecified.  cap = n always suffices.
+ *     meta   2 uint64 out (device): meta[0] = number of pairs (may exceed cap: then only
+ *            cap pairs were written and the caller must retry with a larger cap),
+ *            meta[1] = D.
+ *   Enqueues only (the counts stay on the device).
+ * ecl_cc_merge_encoded: hook the relations of npeers (0..8) encodings into the forest
+ *   `parent` (n entries; does NOT flatten: call ecl_cc_finalize after the last merge).
+ *   bits / pairs / meta / caps are HOST arrays of npeers entries; the buffers they point
+ *   to are device memory readable from the handle's device — local copies, or another
+ *   GPU's buffers mapped with ecl_cc_ipc_open (NVLink peer reads: the transfer happens
+ *   inside the merge kernels).  caps[i] bounds the pairs read from peer i.  The peer
+ *   buffers must stay valid and unchanged until the merge has run on `stream`.
+ * ecl_cc_ipc_export: the ECL_CC_IPC_HANDLE_BYTES-byte handle of a device pointer (CUDA IPC
+ *   handle of its allocation + the pointer's offset in it), for another process.
+ * ecl_cc_ipc_open: map such a handle on `device` (peer access enabled lazily); returns a
+ *   device pointer usable by that process's kernels.  ecl_cc_ipc_close unmaps it.
+ * Errors: INVALID_ARG for bad arguments, ECL_CC_ERR_CUDA when CUDA IPC fails. */
+#define ECL_CC_IPC_HANDLE_BYTES 72
+ECL_CC_API ecl_cc_status ecl_cc_forest_encode(ecl_cc_handle h, int32_t n, const int32_t *labels,
+                                              int32_t anchor, uint32_t *bits, int32_t *pairs,
+                                              int64_t cap, uint64_t *meta, void *stream);
+ECL_CC_API ecl_cc_status ecl_cc_merge_encoded(ecl_cc_handle h, int32_t n, int npeers,
+                                              const uint32_t *const *bits,
+                                              const int32_t *const *pairs,
+                                              const uint64_t *const *meta, const int64_t *caps,
+                                              int32_t *parent, void *stream);
+ECL_CC_API ecl_cc_status ecl_cc_ipc_export(const void *dev_ptr, void *handle_out);
+ECL_CC_API ecl_cc_status ecl_cc_ipc_open(int device, const void *handle, void **dev_ptr_out);
+ECL_CC_API ecl_cc_status ecl_cc_ipc_close(void *dev_ptr);
+
 /* Debug checker (synchronises the stream): offsets monotone with nindex[0]==0 and
  * nindex[n]==m, neighbour IDs in range, graph symmetric.  Returns ECL_CC_OK or
  * ECL_CC_ERR_INVALID_GRAPH.  index_bytes is 4 or 8. */

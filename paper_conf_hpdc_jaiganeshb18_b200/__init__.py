@@ -95,6 +95,12 @@ def _load(stats: bool = False) -> ctypes.CDLL:
             "ecl_cc_io_last_error": ([], ctypes.c_char_p),
             "ecl_cc_merge": ([P, I32, I32, I32, P, P, P], INT),
             "ecl_cc_finalize": ([P, I32, P, P], INT),
+            "ecl_cc_forest_encode": ([P, I32, P, I32, P, P, I64, P, P], INT),
+            "ecl_cc_merge_encoded": ([P, I32, INT, ctypes.POINTER(P), ctypes.POINTER(P),
+                                      ctypes.POINTER(P), ctypes.POINTER(I64), P, P], INT),
+            "ecl_cc_ipc_export": ([P, P], INT),
+            "ecl_cc_ipc_open": ([INT, P, ctypes.POINTER(P)], INT),
+            "ecl_cc_ipc_close": ([P], INT),
             "ecl_cc_validate": ([P, I32, I64, P, INT, P, P], INT),
             "ecl_cc_set_option": ([P, INT, I64], INT),
             "ecl_cc_get_worklist": ([P, P, ctypes.POINTER(I64), P, ctypes.POINTER(I64)], INT),
@@ -112,6 +118,14 @@ def _load(stats: bool = False) -> ctypes.CDLL:
             f.restype = res
         _libs[stats] = lib
         return lib
+
+
+IPC_HANDLE_BYTES = 72   # ECL_CC_IPC_HANDLE_BYTES
+
+
+def _addr(x) -> int:
+    """A device address: a tensor's data pointer or a raw int (e.g. an IPC mapping)."""
+    return x.data_ptr() if isinstance(x, torch.Tensor) else int(x)
 
 
 def _ptr(t: Optional[torch.Tensor]):
@@ -304,6 +318,52 @@ class Handle:
         self._check(self._lib.ecl_cc_finalize(self._h, parent.numel(), _ptr(parent),
                                               _stream_ptr(stream, d)))
         return parent
+
+    # -- encoded forest exchange / P2P merge (ecl_cc_forest_encode, ecl_cc_merge_encoded) --
+    def encode_buffers(self, n: int, cap: Optional[int] = None) -> dict:
+        """Device buffers of one encoding: bits ((n+31)/32 int32 words), pairs (2*cap
+        int32), meta (2 int64: pair count, D)."""
+        d = self.device
+        cap = n if cap is None else cap
+        return {"bits": torch.empty((n + 31) // 32, dtype=torch.int32, device=d),
+                "pairs": torch.empty(2 * max(cap, 1), dtype=torch.int32, device=d),
+                "meta": torch.zeros(2, dtype=torch.int64, device=d), "cap": cap}
+
+    def forest_encode(self, labels: torch.Tensor, anchor: int, enc: dict, stream=None) -> dict:
+        """Encode a flattened labelling as (bitmap of label == labels[anchor], pairs)."""
+        d = self.device
+        _dev_tensor(labels, "labels", (torch.int32,), d)
+        self._check(self._lib.ecl_cc_forest_encode(
+            self._h, labels.numel(), _ptr(labels), int(anchor), _ptr(enc["bits"]),
+            _ptr(enc["pairs"]), int(enc["cap"]), _ptr(enc["meta"]), _stream_ptr(stream, d)))
+        return enc
+
+    def merge_encoded(self, parent: torch.Tensor, peers, stream=None) -> torch.Tensor:
+        """Hook the relations of up to 8 encodings into `parent`.  `peers` is a list of
+        dicts with device pointers or tensors under bits / pairs / meta and an int cap."""
+        d = self.device
+        _dev_tensor(parent, "parent", (torch.int32,), d)
+        k = len(peers)
+        arr = lambda key: (ctypes.c_void_p * max(k, 1))(  # noqa: E731
+            *[_addr(p[key]) for p in peers])
+        caps = (ctypes.c_int64 * max(k, 1))(*[int(p["cap"]) for p in peers])
+        self._check(self._lib.ecl_cc_merge_encoded(
+            self._h, parent.numel(), k, arr("bits"), arr("pairs"), arr("meta"), caps,
+            _ptr(parent), _stream_ptr(stream, d)))
+        return parent
+
+    def ipc_export(self, t: torch.Tensor) -> bytes:
+        buf = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+        self._check(self._lib.ecl_cc_ipc_export(_ptr(t), buf))
+        return buf.raw
+
+    def ipc_open(self, handle: bytes) -> int:
+        out = ctypes.c_void_p()
+        self._check(self._lib.ecl_cc_ipc_open(self.device.index, handle, ctypes.byref(out)))
+        return out.value
+
+    def ipc_close(self, ptr: int):
+        self._check(self._lib.ecl_cc_ipc_close(ctypes.c_void_p(ptr)))
 
     # -- debug ------------------------------------------------------------------------
     def validate(self, nindex: torch.Tensor, nlist: torch.Tensor, stream=None) -> bool:

@@ -281,6 +281,20 @@ ecl_cc_status run_impl(ecl_cc_handle h, int32_t n, int64_t m, const idx_t *ninde
     return st != ECL_CC_OK ? st : se;
 }
 
+// pointers handed out by ecl_cc_ipc_open -> the mapping's base (for ecl_cc_ipc_close)
+std::mutex &ipc_lock()
+{
+    static std::mutex m;
+    return m;
+}
+std::unordered_map<void *, void *> &ipc_bases()
+{
+    static std::unordered_map<void *, void *> b;
+    return b;
+}
+
+typedef int CUresult_compat;   // CUresult (driver API enum; 0 = CUDA_SUCCESS)
+
 }  // namespace
 
 extern "C" {
@@ -423,6 +437,135 @@ ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, int32_t v_h
     }
     CK(cudaGetLastError(), "merge_hook launch");
     return end_call(h, s);
+}
+
+ecl_cc_status ecl_cc_forest_encode(ecl_cc_handle h, int32_t n, const int32_t *labels,
+                                   int32_t anchor, uint32_t *bits, int32_t *pairs,
+                                   int64_t cap, uint64_t *meta, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (n <= 0) return fail_arg(h, "n must be > 0");
+    if (anchor < 0 || anchor >= n) return fail_arg(h, "anchor out of range");
+    if (cap < 0) return fail_arg(h, "cap < 0");
+    if (!labels || !bits || !meta || (cap > 0 && !pairs)) return fail_arg(h, "null pointer");
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    ecl_cc_status st = begin_call(h, s);
+    if (st != ECL_CC_OK) return st;
+    CK(cudaMemsetAsync(meta, 0, sizeof(uint64_t), s), "memset meta");
+    auto k = encode_kernel;
+    const long long words = ((long long)n + kWarp - 1) / kWarp;
+    k<<<grid_for(h, (const void *)k, words * kWarp), kBlock, 0, s>>>(
+        n, labels, anchor, bits, pairs, cap, (unsigned long long *)meta);
+    CK(cudaGetLastError(), "encode launch");
+    return end_call(h, s);
+}
+
+ecl_cc_status ecl_cc_merge_encoded(ecl_cc_handle h, int32_t n, int npeers,
+                                   const uint32_t *const *bits, const int32_t *const *pairs,
+                                   const uint64_t *const *meta, const int64_t *caps,
+                                   int32_t *parent, void *stream)
+{
+    if (!h) return ECL_CC_ERR_INVALID_ARG;
+    if (n <= 0) return fail_arg(h, "n must be > 0");
+    if (npeers < 0 || npeers > kMaxPeers) return fail_arg(h, "npeers must be 0..8");
+    if (!parent || (npeers > 0 && (!bits || !pairs || !meta || !caps)))
+        return fail_arg(h, "null pointer");
+    PeerSet ps{};
+    ps.np = npeers;
+    for (int i = 0; i < npeers; i++) {
+        if (!bits[i] || !meta[i] || caps[i] < 0 || (caps[i] > 0 && !pairs[i]))
+            return fail_arg(h, "null peer buffer");
+        ps.bits[i] = bits[i];
+        ps.pairs[i] = pairs[i];
+        ps.meta[i] = (const unsigned long long *)meta[i];
+        ps.cap[i] = caps[i];
+    }
+    if (npeers == 0) return ECL_CC_OK;
+    DeviceGuard g(h->device);
+    cudaStream_t s = (cudaStream_t)stream;
+    ecl_cc_status st = begin_call(h, s);
+    if (st != ECL_CC_OK) return st;
+    const long long words = ((long long)n + kWarp - 1) / kWarp;
+#ifdef ECL_CC_STATS
+#define ECL_SA , h->cnt + kStatsOff
+#else
+#define ECL_SA
+#endif
+    if (h->load_mode == 1) {
+        auto kb = merge_bits_kernel<1>;
+        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas ECL_SA);
+        auto kp = merge_pairs_kernel<1>;
+        kp<<<grid_for(h, (const void *)kp, -1), kBlock, 0, s>>>(ps, parent, h->ttas ECL_SA);
+    } else {
+        auto kb = merge_bits_kernel<0>;
+        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas ECL_SA);
+        auto kp = merge_pairs_kernel<0>;
+        kp<<<grid_for(h, (const void *)kp, -1), kBlock, 0, s>>>(ps, parent, h->ttas ECL_SA);
+    }
+#undef ECL_SA
+    CK(cudaGetLastError(), "merge_encoded launch");
+    return end_call(h, s);
+}
+
+// CUDA IPC (the peer mappings of the P2P merge): the handle of the allocation holding
+// dev_ptr (cudaIpcGetMemHandle) followed by dev_ptr's byte offset inside it.
+typedef CUresult_compat (*mem_range_fn)(unsigned long long *, size_t *, unsigned long long);
+
+ecl_cc_status ecl_cc_ipc_export(const void *dev_ptr, void *handle_out)
+{
+    if (!dev_ptr || !handle_out) return ECL_CC_ERR_INVALID_ARG;
+    static mem_range_fn range = nullptr;
+    if (!range) {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess || !fn)
+            return ECL_CC_ERR_CUDA;
+        range = (mem_range_fn)fn;
+    }
+    unsigned long long base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (unsigned long long)(uintptr_t)dev_ptr) != 0) return ECL_CC_ERR_CUDA;
+    cudaIpcMemHandle_t mh;
+    if (cudaIpcGetMemHandle(&mh, (void *)(uintptr_t)base) != cudaSuccess) return ECL_CC_ERR_CUDA;
+    const uint64_t off = (uint64_t)((uintptr_t)dev_ptr - base);
+    memcpy(handle_out, &mh, sizeof(mh));
+    memcpy((char *)handle_out + sizeof(mh), &off, sizeof(off));
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_ipc_open(int device, const void *handle, void **dev_ptr_out)
+{
+    if (!handle || !dev_ptr_out) return ECL_CC_ERR_INVALID_ARG;
+    *dev_ptr_out = nullptr;
+    DeviceGuard g(device);
+    if (!g.ok) return ECL_CC_ERR_INVALID_ARG;
+    cudaIpcMemHandle_t mh;
+    uint64_t off = 0;
+    memcpy(&mh, handle, sizeof(mh));
+    memcpy(&off, (const char *)handle + sizeof(mh), sizeof(off));
+    void *base = nullptr;
+    if (cudaIpcOpenMemHandle(&base, mh, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+        return ECL_CC_ERR_CUDA;
+    std::lock_guard<std::mutex> lk(ipc_lock());
+    ipc_bases()[(char *)base + off] = base;
+    *dev_ptr_out = (char *)base + off;
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_ipc_close(void *dev_ptr)
+{
+    if (!dev_ptr) return ECL_CC_ERR_INVALID_ARG;
+    void *base = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(ipc_lock());
+        auto it = ipc_bases().find(dev_ptr);
+        if (it == ipc_bases().end()) return ECL_CC_ERR_INVALID_ARG;
+        base = it->second;
+        ipc_bases().erase(it);
+    }
+    return cudaIpcCloseMemHandle(base) == cudaSuccess ? ECL_CC_OK : ECL_CC_ERR_CUDA;
 }
 
 ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream)

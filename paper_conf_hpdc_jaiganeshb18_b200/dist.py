@@ -144,6 +144,133 @@ def forest_merge(parent: torch.Tensor, ops, group=None, chunks: int = 4,
     return parent if rank == 0 else None
 
 
+def row_anchor(nindex_rows: torch.Tensor, lo: int) -> int:
+    """The highest-degree row of a slice (the encoding's anchor: its label is normally the
+    rank's giant component, so the bitmap holds most vertices and the pair list is
+    short)."""
+    deg = (nindex_rows[1:] - nindex_rows[:-1]).to(torch.int64)
+    return lo + (int(torch.argmax(deg)) if deg.numel() else 0)
+
+
+class EncodedMerge:
+    """Flat merge of encoded forests into rank 0 (the variants the survey
+    lists beside the binomial tree of full forests).
+
+    Every rank g != 0 flattens its local forest (ecl_cc_finalize), encodes it
+    (ecl_cc_forest_encode: an n/32-word bitmap of "label == D" plus the pairs (v, L[v]) of
+    the remaining non-roots — for a power-law graph 16 MB + a few MB instead of the 537 MB
+    label array at n = 2^27), and rank 0 hooks all peers' relations in one
+    ecl_cc_merge_encoded call, then flattens once.  Exact by hook-once sufficiency
+    (P:L161-L163): the encoded edges span the same classes as the labels.
+
+    mode "compact": the encodings travel over the process group (NCCL send/recv; gloo
+      stages through host memory).  The pair count is exchanged first (one small host
+      synchronisation per step) so only the used part of the pair buffer is sent.
+    mode "p2p": no copies.  Each rank exports its encoding buffers once (CUDA IPC,
+      ecl_cc_ipc_export); rank 0 maps them (ecl_cc_ipc_open) and its merge kernels read
+      the peers' bitmaps and pairs directly over NVLink, so the transfer happens inside the
+      merge.  The process group only orders the steps: a one-int "encoded" signal from
+      every peer before the merge and an "done reading" acknowledgement back after it.
+      With NCCL both are stream-ordered device operations (no host synchronisation); with
+      gloo (tests, one GPU) the streams are synchronised around host messages.
+    """
+
+    def __init__(self, handle, n: int, anchor: int, mode: str = "p2p", group=None):
+        if mode not in ("compact", "p2p"):
+            raise ValueError(mode)
+        self.h, self.n, self.anchor, self.mode, self.group = handle, n, anchor, mode, group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        if self.world - 1 > 8:
+            raise ValueError("EncodedMerge merges at most 8 peers into rank 0")
+        self.gloo = dist.get_backend(group) == "gloo"
+        dev = handle.device
+        self.flag = torch.ones(1, dtype=torch.int32, device=dev)
+        self.enc = handle.encode_buffers(n) if self.rank != 0 else None
+        self.peers = []
+        self.mapped = []
+        if mode == "p2p":
+            hs = None
+            if self.rank != 0:
+                hs = {k: handle.ipc_export(self.enc[k]) for k in ("bits", "pairs", "meta")}
+            allh = [None] * self.world
+            dist.all_gather_object(allh, hs, group=group)
+            if self.rank == 0:
+                for r in range(1, self.world):
+                    ptrs = {k: handle.ipc_open(allh[r][k]) for k in ("bits", "pairs", "meta")}
+                    self.mapped += list(ptrs.values())
+                    self.peers.append({**ptrs, "cap": n})
+        elif self.rank == 0:
+            self.recv = [handle.encode_buffers(n) for _ in range(1, self.world)]
+
+    def close(self):
+        for p in self.mapped:
+            self.h.ipc_close(p)
+        self.mapped = []
+
+    # -- transport helpers (NCCL: stream-ordered device ops; gloo: host messages) --------
+    def _send(self, t, dst):
+        if self.gloo and t.is_cuda:
+            t = t.cpu()                       # synchronises the stream first
+        dist.send(t, dst=_g(self.group, dst), group=self.group)
+
+    def _recv(self, t, src):
+        if self.gloo and t.is_cuda:
+            host = torch.empty(t.shape, dtype=t.dtype)
+            dist.recv(host, src=_g(self.group, src), group=self.group)
+            t.copy_(host)
+        else:
+            dist.recv(t, src=_g(self.group, src), group=self.group)
+
+    def __call__(self, parent: torch.Tensor, broadcast: bool = False):
+        h, rank = self.h, self.rank
+        if self.world == 1:
+            h.finalize(parent)
+        elif rank != 0:
+            h.finalize(parent)                              # labels = roots
+            h.forest_encode(parent, self.anchor, self.enc)
+            if self.mode == "p2p":
+                self._send(self.flag, 0)                    # "my encoding is complete"
+                self._recv(self.flag, 0)                    # rank 0 finished reading it
+            else:
+                meta = self.enc["meta"]
+                self._send(meta, 0)
+                npairs = int(meta[0].item())
+                self._send(self.enc["bits"], 0)
+                if npairs:
+                    self._send(self.enc["pairs"][:2 * npairs], 0)
+        else:
+            if self.mode == "p2p":
+                for r in range(1, self.world):
+                    self._recv(self.flag, r)
+                h.merge_encoded(parent, self.peers)
+                if self.gloo:
+                    torch.cuda.current_stream(parent.device).synchronize()
+                for r in range(1, self.world):
+                    self._send(self.flag, r)
+            else:
+                peers = []
+                for r, buf in zip(range(1, self.world), self.recv):
+                    self._recv(buf["meta"], r)
+                    npairs = int(buf["meta"][0].item())
+                    self._recv(buf["bits"], r)
+                    if npairs:
+                        self._recv(buf["pairs"][:2 * npairs], r)
+                    peers.append({"bits": buf["bits"], "pairs": buf["pairs"],
+                                  "meta": buf["meta"], "cap": npairs})
+                h.merge_encoded(parent, peers)
+            h.finalize(parent)
+        if broadcast:
+            if self.gloo and parent.is_cuda:
+                host = parent.cpu()
+                dist.broadcast(host, src=_g(self.group, 0), group=self.group)
+                parent.copy_(host)
+            else:
+                dist.broadcast(parent, src=_g(self.group, 0), group=self.group)
+            return parent
+        return parent if rank == 0 else None
+
+
 def _g(group, r):
     return r if group is None else dist.get_global_rank(group, r)
 

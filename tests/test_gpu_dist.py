@@ -57,7 +57,12 @@ def _worker(rank, world, port, name, sd, seed, chunks, broadcast, loopdup, varia
             if variant == "tree":
                 out = edist.forest_merge(parent, h, chunks=chunks, broadcast=broadcast)
             else:
-                out = edist.forest_merge_variant(parent, h, variant, broadcast=broadcast)
+                mg = edist.EncodedMerge(h, n, edist.row_anchor(idx, lo), mode=variant)
+                for _ in range(2):        # twice: buffers and mappings are reused per step
+                    p2 = h.run_rows(n, lo, hi, idx, lst, flatten=False)
+                    out = mg(p2, broadcast=broadcast)
+                torch.cuda.synchronize()
+                mg.close()
             torch.cuda.synchronize()
             q.put((rank, None if out is None else out.cpu().numpy().copy()))
     except Exception as e:       # surface the error in the parent
@@ -106,3 +111,18 @@ def test_multiprocess_tree_merge_broadcast(name, sd):
 def test_multiprocess_raw_csr():
     # self-loops and duplicate entries through the distributed path as well
     run_world(3, "C4", 8, seed=5, loopdup=True)
+
+
+@pytest.mark.parametrize("variant", ["compact", "p2p"])
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("name,sd", [("C4", 7), ("C5", 10), ("C2", 6)])
+def test_multiprocess_encoded_merge(variant, world, name, sd):
+    """Encoded forests (bitmap of the anchor's class + pairs) merged into rank 0: sent over
+    the process group ("compact") or read by rank 0's merge kernels straight from the
+    peers' memory through CUDA IPC mappings ("p2p")."""
+    run_world(world, name, sd, seed=world + 10, variant=variant)
+
+
+@pytest.mark.parametrize("variant", ["compact", "p2p"])
+def test_multiprocess_encoded_merge_broadcast_raw(variant):
+    run_world(3, "C4", 8, seed=21, broadcast=True, loopdup=True, variant=variant)

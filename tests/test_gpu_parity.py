@@ -472,3 +472,69 @@ def test_cuda_graph_capture_replay(h, name, order):
             assert np.array_equal(out.cpu().numpy(), expect)
     finally:
         h.set_option("order", DEFAULTS["order"])
+
+
+# ---------------------------------------------------------------------------------------
+# encoded forest exchange: encode each fake rank's flattened forest,
+# merge all encodings into rank 0's forest in one call, flatten once
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("G", [2, 3, 5, 9])
+@pytest.mark.parametrize("name", ["C2", "C4", "C5"])
+def test_fake_multi_gpu_encoded_merge(h, name, G):
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config(name, seed=7, scale_down=SMALL[name] + 1, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64, G, weights=dist.row_weights(nindex64, g.nlist))
+    forests, encs = [], []
+    for r in range(G):
+        idx, lst = dist.slice_rows(nindex64, g.nlist, bounds[r], bounds[r + 1])
+        f = h.run_rows(g.n, bounds[r], bounds[r + 1], idx, lst, flatten=(r > 0))
+        forests.append(f)
+        if r > 0:
+            enc = h.encode_buffers(g.n)
+            h.forest_encode(f, dist.row_anchor(idx, bounds[r]), enc)
+            encs.append(enc)
+    h.merge_encoded(forests[0], encs)
+    h.finalize(forests[0])
+    torch.cuda.synchronize()
+    assert np.array_equal(forests[0].cpu().numpy(), expect)
+
+
+def test_forest_encode_exact(h):
+    """The encoding of a flattened labelling: bitmap = {v : L[v] == L[anchor]}, pairs =
+    {(v, L[v]) : L[v] != v, L[v] != D}, meta = (#pairs, D)."""
+    g = gg.make_config("C4", seed=8, scale_down=8, device="cuda")
+    lab = h.run(g.nindex, g.nlist)
+    anchor = int(torch.argmax(g.degrees()))
+    enc = h.encode_buffers(g.n)
+    h.forest_encode(lab, anchor, enc)
+    torch.cuda.synchronize()
+    L = lab.cpu().numpy()
+    D = L[anchor]
+    meta = enc["meta"].cpu().numpy()
+    assert meta[1] == D
+    v = np.arange(g.n)
+    want_pairs = set(zip(v[(L != v) & (L != D)].tolist(), L[(L != v) & (L != D)].tolist()))
+    P = enc["pairs"].cpu().numpy()[:2 * meta[0]].reshape(-1, 2)
+    assert meta[0] == len(want_pairs) and set(map(tuple, P.tolist())) == want_pairs
+    bits = enc["bits"].cpu().numpy().view(np.uint32)
+    got = (bits[v // 32] >> (v % 32)) & 1
+    assert np.array_equal(got.astype(bool), L == D)
+    # merging the encoding into an identity forest and flattening reproduces the labels
+    par = torch.arange(g.n, dtype=torch.int32, device="cuda")
+    h.merge_encoded(par, [enc])
+    h.finalize(par)
+    assert np.array_equal(par.cpu().numpy(), L)
+
+
+def test_forest_encode_small_cap(h):
+    """meta[0] reports the needed pair count when cap is too small (only cap written)."""
+    g = gg.make_config("C1", seed=9, device="cuda")
+    lab = h.run(g.nindex, g.nlist)
+    enc = h.encode_buffers(g.n, cap=3)
+    h.forest_encode(lab, 0, enc)
+    L = lab.cpu().numpy()
+    D = L[0]
+    v = np.arange(g.n)
+    assert int(enc["meta"][0]) == int(((L != v) & (L != D)).sum()) > 3

@@ -12,6 +12,14 @@ of rounds + rank 0's finalize.  The merged labels are checked against the single
 labels.  --even uses the plain m/G entry split instead of the work-weighted one.
 
     python tools/mgpu_emulate.py [--config C5] [--gpus 1,2,4,8] [--link-gbs 750] [--order 2]
+                                 [--merge tree,encoded]
+
+--merge encoded projects dist.EncodedMerge: every rank g > 0 flattens
+its local forest and encodes it (ecl_cc_forest_encode: bitmap of its anchor's class +
+pairs), rank 0 merges all encodings in one ecl_cc_merge_encoded call (kernels timed here
+on local copies) and flattens once.  In the p2p mode the merge kernels read the peers'
+buffers over NVLink, so the merge is modelled as max(kernel time, encoded bytes / link
+bandwidth into rank 0); the compact mode adds the transfer instead.
 """
 import argparse
 import json
@@ -39,6 +47,80 @@ def timed(fn, reps=3):
     return best, out
 
 
+def tree_merge(h, forests, G, n, args, ref, t_rank):
+    rounds = {}
+    for (rd, send, recv) in edist.tree_schedule(G):
+        base = forests[recv].clone()
+
+        def mrg():
+            forests[recv].copy_(base)
+            h.merge(forests[recv], forests[send])
+            return None
+        copy_t, _ = timed(lambda: forests[recv].copy_(base))
+        t_m, _ = timed(mrg)
+        t_m = max(t_m - copy_t, 0.0)
+        forests[recv].copy_(base)
+        h.merge(forests[recv], forests[send])
+        xfer = n * 4 / (args.link_gbs * 1e9) * 1e3
+        rt = xfer + t_m / args.chunks
+        rounds.setdefault(rd, []).append({"send": send, "recv": recv, "merge_ms": round(t_m, 4),
+                                          "transfer_ms_model": round(xfer, 4),
+                                          "round_ms": round(rt, 4)})
+        del base
+    t_fin, _ = timed(lambda: h.finalize(forests[0]), reps=1)
+    torch.cuda.synchronize()
+    ok = bool(torch.equal(forests[0], ref))
+    t_rounds = sum(max(x["round_ms"] for x in v) for v in rounds.values())
+    return {"merge_rounds": rounds, "final_flatten_ms": round(t_fin, 4),
+            "merge_total_ms": round(t_rounds + t_fin, 4), "labels_exact": ok,
+            "projected_ms": round(max(t_rank) + t_rounds + t_fin, 4)}
+
+
+def encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank):
+    """Flatten + encode on every rank g > 0, one merge of all encodings into rank 0."""
+    encs, t_prep, pair_counts = [], [], []
+    for r in range(1, G):
+        idx = nidx64[bounds[r]:bounds[r + 1] + 1]
+        anchor = edist.row_anchor(idx, bounds[r])
+        enc = h.encode_buffers(n)
+        f = forests[r].clone()
+
+        def prep():
+            f.copy_(forests[r])
+            h.finalize(f)
+            h.forest_encode(f, anchor, enc)
+        t_copy, _ = timed(lambda: f.copy_(forests[r]))
+        t, _ = timed(prep)
+        t_prep.append(max(t - t_copy, 0.0))
+        pair_counts.append(int(enc["meta"][0]))
+        encs.append(enc)
+        del f
+    base = forests[0].clone()
+
+    def mrg():
+        forests[0].copy_(base)
+        h.merge_encoded(forests[0], encs)
+    copy_t, _ = timed(lambda: forests[0].copy_(base))
+    t_m, _ = timed(mrg)
+    t_m = max(t_m - copy_t, 0.0)
+    forests[0].copy_(base)
+    h.merge_encoded(forests[0], encs)
+    t_fin, _ = timed(lambda: h.finalize(forests[0]), reps=1)
+    torch.cuda.synchronize()
+    ok = bool(torch.equal(forests[0], ref))
+    enc_bytes = sum(((n + 31) // 32) * 4 + 16 + 8 * c for c in pair_counts)
+    xfer = enc_bytes / (args.link_gbs * 1e9) * 1e3
+    ready = max([t_rank[0]] + [t_rank[r] + t_prep[r - 1] for r in range(1, G)])
+    p2p = ready + max(t_m, xfer) + t_fin
+    compact = ready + xfer + t_m + t_fin
+    return {"prep_ms": [round(x, 4) for x in t_prep], "pairs": pair_counts,
+            "encoded_bytes_total": enc_bytes, "merge_ms": round(t_m, 4),
+            "transfer_ms_model": round(xfer, 4), "final_flatten_ms": round(t_fin, 4),
+            "merge_total_p2p_ms": round(max(t_m, xfer) + t_fin, 4),
+            "projected_ms": round(p2p, 4), "projected_compact_ms": round(compact, 4),
+            "labels_exact": ok}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C5")
@@ -47,6 +129,7 @@ def main():
     ap.add_argument("--chunks", type=int, default=4)
     ap.add_argument("--even", action="store_true")
     ap.add_argument("--order", type=int, default=2, help="ECL_CC_OPT_ORDER of every run")
+    ap.add_argument("--merge", default="tree,encoded")
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=1, device="cuda")
     n, m = g.n, g.m
@@ -71,37 +154,19 @@ def main():
             t_rank.append(t)
             forests.append(par)
             del idx, lst
-        rounds = {}
-        for (rd, send, recv) in edist.tree_schedule(G):
-            base = forests[recv].clone()
-
-            def mrg():
-                forests[recv].copy_(base)
-                h.merge(forests[recv], forests[send])
-                return None
-            copy_t, _ = timed(lambda: forests[recv].copy_(base))
-            t_m, _ = timed(mrg)
-            t_m = max(t_m - copy_t, 0.0)
-            forests[recv].copy_(base)
-            h.merge(forests[recv], forests[send])
-            xfer = n * 4 / (args.link_gbs * 1e9) * 1e3
-            rt = xfer + t_m / args.chunks
-            rounds.setdefault(rd, []).append({"send": send, "recv": recv, "merge_ms": round(t_m, 4),
-                                              "transfer_ms_model": round(xfer, 4),
-                                              "round_ms": round(rt, 4)})
-            del base
-        t_fin = 0.0
-        if G > 1:
-            t_fin, _ = timed(lambda: h.finalize(forests[0]), reps=1)
-        torch.cuda.synchronize()
-        ok = bool(torch.equal(forests[0], ref))
-        t_rounds = sum(max(x["round_ms"] for x in v) for v in rounds.values())
-        proj = max(t_rank) + t_rounds + t_fin
-        res["rows"].append({"gpus": G, "rank_forest_ms": [round(x, 4) for x in t_rank],
-                            "merge_rounds": rounds, "final_flatten_ms": round(t_fin, 4),
-                            "projected_ms": round(proj, 4),
-                            "projected_Medges_s": round(m / proj / 1e3, 1),
-                            "projected_speedup": round(t1 / proj, 3), "labels_exact": ok})
+        row = {"gpus": G, "rank_forest_ms": [round(x, 4) for x in t_rank]}
+        if "tree" in args.merge and G > 1:
+            tf = [f.clone() for f in forests]
+            row["tree"] = tree_merge(h, tf, G, n, args, ref, t_rank)
+            del tf
+        if "encoded" in args.merge and G > 1:
+            row["encoded"] = encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank)
+        if G == 1:
+            row["projected_ms"] = round(t_rank[0], 4)
+        best = min([row[k]["projected_ms"] for k in ("tree", "encoded") if k in row] or
+                   [row.get("projected_ms", t_rank[0])])
+        row["projected_speedup_best"] = round(t1 / best, 3)
+        res["rows"].append(row)
         del forests
         torch.cuda.empty_cache()
     print(json.dumps(res))

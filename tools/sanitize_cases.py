@@ -42,6 +42,8 @@ def cases(quick):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--variants", action="store_true",
+                    help="also the ablation paths (Jump1-3, batch 0, Init1/2, Fini1/2)")
     args = ap.parse_args()
     bad = 0
     runs = 0
@@ -62,6 +64,19 @@ def main():
                                 print(f"MISMATCH {g.name} order={order} prejump={prejump} "
                                       f"filter={filt} idx={idx.dtype}", flush=True)
                                 bad += 1
+            if args.variants:
+                for opts in (dict(jump=1), dict(jump=2), dict(jump=3), dict(batch=0),
+                             dict(init=1, fini=1), dict(init=2, fini=2)):
+                    for k, v in opts.items():
+                        h.set_option(k, v)
+                    out = h.run(gd.nindex, gd.nlist)
+                    torch.cuda.synchronize()
+                    runs += 1
+                    if not np.array_equal(out.cpu().numpy(), expect):
+                        print(f"MISMATCH {g.name} {opts}", flush=True)
+                        bad += 1
+                    for k in opts:
+                        h.set_option(k, {"jump": 4, "batch": 1, "init": 3, "fini": 3}[k])
             h.set_option("order", 2).set_option("prejump", 1).set_option("filter", 2)
             lab, ta, tb = h.spanning_forest(gd.nindex, gd.nlist)
             torch.cuda.synchronize()
@@ -77,6 +92,7 @@ def main():
             for r in range(3):
                 i, l_ = edist.slice_rows(nidx64, gd.nlist, b[r], b[r + 1])
                 forests.append(h.run_rows(g.n, b[r], b[r + 1], i, l_, flatten=False))
+            f0 = forests[0].clone()
             for (_, s, rcv) in edist.tree_schedule(3):
                 h.merge(forests[rcv], forests[s])
             h.finalize(forests[0])
@@ -84,6 +100,21 @@ def main():
             runs += 1
             if not np.array_equal(forests[0].cpu().numpy(), expect):
                 print(f"MERGE MISMATCH {g.name}", flush=True)
+                bad += 1
+            # encoded merge of ranks 1, 2 into rank 0
+            encs = []
+            for r in (1, 2):
+                i, l_ = edist.slice_rows(nidx64, gd.nlist, b[r], b[r + 1])
+                f = h.run_rows(g.n, b[r], b[r + 1], i, l_)
+                e = h.encode_buffers(g.n)
+                h.forest_encode(f, edist.row_anchor(i, b[r]), e)
+                encs.append(e)
+            h.merge_encoded(f0, encs)
+            h.finalize(f0)
+            torch.cuda.synchronize()
+            runs += 1
+            if not np.array_equal(f0.cpu().numpy(), expect):
+                print(f"ENCODED MERGE MISMATCH {g.name}", flush=True)
                 bad += 1
     print(f"sanitize_cases: {runs} runs, {bad} mismatches", flush=True)
     sys.exit(1 if bad else 0)
