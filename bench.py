@@ -348,13 +348,15 @@ def launches_per_step(world: int, rank: int, chunks: int, merge: str) -> int:
     """Our kernels per step on `rank`: init_bin, depth_probe, prejump (exits at once on
     shallow forests), hook_thread, hook_range x2, finalize; with G ranks: identity_outside
     instead of finalize in run_rows, then for the tree merge one merge_hook per received
-    chunk and rank 0's finalize, for the encoded merges finalize + encode on every rank
-    g > 0 and merge_bits + merge_pairs + finalize on rank 0."""
+    chunk and rank 0's finalize; for the encoded merges a flatten (R23 depth probe +
+    passes + finalize) and encode on every rank g > 0, and on rank 0 a flatten,
+    merge_bits + merge_pairs, and a flatten."""
     if world == 1:
         return 7
-    if merge != "tree":
-        return 7 + (3 if rank == 0 else 2)
     from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
+    if merge != "tree":
+        fl = 3 if edist.EncodedMerge.FLATTEN.get("flatten_passes") else 1
+        return 7 + (2 * fl + 2 if rank == 0 else fl + 1)
     recv = sum(1 for (_, _s, r) in edist.tree_schedule(world) if r == rank)
     return 7 + recv * chunks + (1 if rank == 0 else 0)
 

@@ -187,7 +187,8 @@ ECL_CC_API ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *pa
  * ecl_cc_forest_encode: encode a FLATTENED labelling `labels` (n entries, labels[v] the
  *   root of v's tree, e.g. the output of ecl_cc_run_rows without STOP_AFTER 2, or of
  *   ecl_cc_finalize) as the relation it spans: D = labels[anchor] (pick a vertex of the
- *   largest component, e.g. the highest-degree row), bits[v / 32] bit v % 32 set iff
+ *   largest component, e.g. the highest-degree row; anchor = -1: no bitmap class, every
+ *   non-root becomes a pair), bits[v / 32] bit v % 32 set iff
  *   labels[v] == D, and the pairs (v, labels[v]) of every other v with labels[v] != v.
  *   The edges {(v, D) : bit v} u {(v, labels[v]) : pairs} span exactly the classes of
  *   `labels`, so merging them is exact (hook-once sufficiency).
@@ -270,12 +271,17 @@ typedef enum {
                                      then warp on the run's stream with full grids that
                                      take the SM slots hook_block leaves or retires.
                                      Labels are the same in every order (R13).         */
-    ECL_CC_OPT_PREJUMP = 17       /* pointer-doubling passes between init and the hook
+    ECL_CC_OPT_PREJUMP = 17,      /* pointer-doubling passes between init and the hook
                                      kernels (R23; Jump's pointer jumping,
                                      P:L245, as synchronous passes): 0 off, 1 always,
                                      2 (default) only when a sample of the Init3
                                      forest is deep (meshes, road-like graphs).
                                      Labels are unchanged (R13).                       */
+    ECL_CC_OPT_FLATTEN_PASSES = 18 /* ecl_cc_finalize only: run R23's pointer-jumping
+                                     passes before the finalize kernel: 0 (default) off,
+                                     1 always, 2 when a depth probe finds the forest deep.
+                                     For merged multi-GPU forests, whose former roots
+                                     form long chains that Fini3 would walk per vertex. */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 
@@ -295,7 +301,11 @@ ECL_CC_API ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4]);
  * (u == parent[v] or u == v_rep), [6] checked against the R21 bitmap, [7] skipped by the
  * bitmap, [8] hop-1 gathers parent[u], [9] hop-2 gathers, [10] bitmap marks,
  * [11] non-empty edge windows (process_window calls), [12] edges deferred to the R22
- * hook queue.  Others are 0. */
+ * hook queue, and the path lengths of the find_repres walks (Table 4 analogue,
+ * P:L329-L337; length = parent pointers followed from the walk's start to where it
+ * stopped — the root, or v_rep under the early exit; walks from a root are not counted,
+ * nor edges the R21/R22 probe settles without a walk): [13] sum of lengths, [14] walks,
+ * [15] maximum length. */
 ECL_CC_API ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int count);
 
 /* Per-phase device time of the most recent full run with ECL_CC_OPT_TIMING set

@@ -45,6 +45,7 @@ OPT = {
     "filter": 15,
     "order": 16,
     "prejump": 17,
+    "flatten_passes": 18,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 
@@ -396,7 +397,8 @@ class Handle:
 
     STAT_NAMES = ("cas_success", "cas_fail", "finds", "halving_stores", "edges_v_gt_u",
                   "edges_r15_same_tree", "edges_bitmap_checked", "edges_bitmap_skipped",
-                  "gathers_hop1", "gathers_hop2", "bitmap_marks", "windows", "edges_queued")
+                  "gathers_hop1", "gathers_hop2", "bitmap_marks", "windows", "edges_queued",
+                  "path_len_sum", "find_walks", "path_len_max")
 
     def stats(self) -> dict:
         """ECL_CC_STATS counters of the last run (ecl_cc_get_stats_ex)."""

@@ -445,7 +445,7 @@ ecl_cc_status ecl_cc_forest_encode(ecl_cc_handle h, int32_t n, const int32_t *la
 {
     if (!h) return ECL_CC_ERR_INVALID_ARG;
     if (n <= 0) return fail_arg(h, "n must be > 0");
-    if (anchor < 0 || anchor >= n) return fail_arg(h, "anchor out of range");
+    if (anchor < -1 || anchor >= n) return fail_arg(h, "anchor out of range");
     if (cap < 0) return fail_arg(h, "cap < 0");
     if (!labels || !bits || !meta || (cap > 0 && !pairs)) return fail_arg(h, "null pointer");
     DeviceGuard g(h->device);
@@ -578,6 +578,21 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
     cudaStream_t s = (cudaStream_t)stream;
     ecl_cc_status st = begin_call(h, s);
     if (st != ECL_CC_OK) return st;
+    if (h->flatten_passes) {
+        // R23's synchronous pointer-jumping passes first (forests merged from several
+        // ranks can hold long chains of former roots, which Fini3 would walk per vertex)
+        int *ctl = (int *)(h->cnt + 4);
+        CK(cudaMemsetAsync(ctl, 0, 4 * sizeof(unsigned long long), s), "memset ctl");
+        depth_probe_kernel<<<1, kBlock, 0, s>>>(0, n, parent, ctl, h->flatten_passes);
+        auto k = prejump_kernel;
+        const int blocks = std::min(h->sms * blocks_per_sm(h, (const void *)k, 0),
+                                    (int)std::max(1LL, ((long long)n + kBlock - 1) / kBlock));
+        int a0 = 0, a1 = n;
+        int *a2 = parent, *a3 = ctl;
+        void *args[] = {&a0, &a1, &a2, &a3};
+        CK(cudaLaunchCooperativeKernel((const void *)k, dim3(blocks), dim3(kBlock), args, 0, s),
+           "flatten passes launch");
+    }
     if (h->fini == 3 && kFastFini) {
         auto k = finalize3_kernel<0>;
         k<<<grid_for(h, (const void *)k, ((long long)n + kFinPer - 1) / kFinPer), kBlock, 0, s>>>(n, parent);
@@ -754,6 +769,10 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_PREJUMP:
         if (value < 0 || value > 2) return fail_arg(h, "prejump must be 0, 1 or 2");
         h->prejump = (int)value;
+        break;
+    case ECL_CC_OPT_FLATTEN_PASSES:
+        if (value < 0 || value > 2) return fail_arg(h, "flatten_passes must be 0, 1 or 2");
+        h->flatten_passes = (int)value;
         break;
     case ECL_CC_OPT_BATCH:
         h->batch = value != 0;

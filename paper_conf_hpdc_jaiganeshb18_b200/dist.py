@@ -149,7 +149,7 @@ def row_anchor(nindex_rows: torch.Tensor, lo: int) -> int:
     rank's giant component, so the bitmap holds most vertices and the pair list is
     short)."""
     deg = (nindex_rows[1:] - nindex_rows[:-1]).to(torch.int64)
-    return lo + (int(torch.argmax(deg)) if deg.numel() else 0)
+    return lo + int(torch.argmax(deg)) if deg.numel() else -1     # -1: empty slice
 
 
 class EncodedMerge:
@@ -175,10 +175,18 @@ class EncodedMerge:
       gloo (tests, one GPU) the streams are synchronised around host messages.
     """
 
-    def __init__(self, handle, n: int, anchor: int, mode: str = "p2p", group=None):
+    # ecl_cc_finalize options of the flattens: a local forest's vertices outside the rank's
+    # rows hang below chains of former roots (each hooked once, never walked again), so a
+    # plain Fini3 walk per vertex is slow; the R23 pointer-jumping passes first shorten
+    # every chain (ECL_CC_OPT_FLATTEN_PASSES)
+    FLATTEN = {"fini": 3, "flatten_passes": 1}
+
+    def __init__(self, handle, n: int, anchor: int, mode: str = "p2p", group=None,
+                 flatten: Optional[dict] = None):
         if mode not in ("compact", "p2p"):
             raise ValueError(mode)
         self.h, self.n, self.anchor, self.mode, self.group = handle, n, anchor, mode, group
+        self.flatten = dict(self.FLATTEN if flatten is None else flatten)
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
         if self.world - 1 > 8:
@@ -203,6 +211,14 @@ class EncodedMerge:
         elif self.rank == 0:
             self.recv = [handle.encode_buffers(n) for _ in range(1, self.world)]
 
+    def _flatten(self, parent):
+        for k, v in self.flatten.items():
+            self.h.set_option(k, v)
+        try:
+            self.h.finalize(parent)
+        finally:
+            self.h.set_option("fini", 3).set_option("flatten_passes", 0)
+
     def close(self):
         for p in self.mapped:
             self.h.ipc_close(p)
@@ -225,9 +241,9 @@ class EncodedMerge:
     def __call__(self, parent: torch.Tensor, broadcast: bool = False):
         h, rank = self.h, self.rank
         if self.world == 1:
-            h.finalize(parent)
+            self._flatten(parent)
         elif rank != 0:
-            h.finalize(parent)                              # labels = roots
+            self._flatten(parent)                           # labels = roots
             h.forest_encode(parent, self.anchor, self.enc)
             if self.mode == "p2p":
                 self._send(self.flag, 0)                    # "my encoding is complete"
@@ -240,6 +256,7 @@ class EncodedMerge:
                 if npairs:
                     self._send(self.enc["pairs"][:2 * npairs], 0)
         else:
+            self._flatten(parent)              # the merge's finds are then one hop long
             if self.mode == "p2p":
                 for r in range(1, self.world):
                     self._recv(self.flag, r)
@@ -259,7 +276,7 @@ class EncodedMerge:
                     peers.append({"bits": buf["bits"], "pairs": buf["pairs"],
                                   "meta": buf["meta"], "cap": npairs})
                 h.merge_encoded(parent, peers)
-            h.finalize(parent)
+            self._flatten(parent)
         if broadcast:
             if self.gloo and parent.is_cuda:
                 host = parent.cpu()

@@ -538,3 +538,43 @@ def test_forest_encode_small_cap(h):
     D = L[0]
     v = np.arange(g.n)
     assert int(enc["meta"][0]) == int(((L != v) & (L != D)).sum()) > 3
+
+
+@pytest.mark.parametrize("passes", [1, 2])
+@pytest.mark.parametrize("name", ["C2", "C5"])
+def test_finalize_with_flatten_passes(h, name, passes):
+    """ecl_cc_finalize with R23's passes first (ECL_CC_OPT_FLATTEN_PASSES) on unflattened
+    local forests merged along the tree: same labels."""
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config(name, seed=11, scale_down=SMALL[name] + 1, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64, 4)
+    forests = []
+    for r in range(4):
+        idx, lst = dist.slice_rows(nindex64, g.nlist, bounds[r], bounds[r + 1])
+        forests.append(h.run_rows(g.n, bounds[r], bounds[r + 1], idx, lst, flatten=False))
+    for (_, send, recv) in dist.tree_schedule(4):
+        h.merge(forests[recv], forests[send])
+    h.set_option("flatten_passes", passes)
+    try:
+        h.finalize(forests[0])
+        torch.cuda.synchronize()
+    finally:
+        h.set_option("flatten_passes", 0)
+    assert np.array_equal(forests[0].cpu().numpy(), expect)
+
+
+def test_path_length_counters():
+    """Table 4 analogue counters (stats build): every counted walk follows >= 1 pointer,
+    the maximum bounds the average, and Jump3 (no compression) walks at least as far."""
+    with ecl.Handle(0, stats=True) as hs:
+        g = gg.make_config("C2", seed=1, scale_down=6, device="cuda")
+        res = {}
+        for jump in (4, 3):
+            gpu_labels(hs, g, jump=jump)
+            st = hs.stats()
+            assert st["find_walks"] > 0 and st["path_len_max"] >= 1
+            assert st["find_walks"] <= st["path_len_sum"] <= st["path_len_max"] * st["find_walks"]
+            res[jump] = st["path_len_sum"] / st["find_walks"]
+        assert res[3] >= res[4]

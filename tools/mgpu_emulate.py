@@ -67,53 +67,87 @@ def tree_merge(h, forests, G, n, args, ref, t_rank):
                                           "transfer_ms_model": round(xfer, 4),
                                           "round_ms": round(rt, 4)})
         del base
-    t_fin, _ = timed(lambda: h.finalize(forests[0]), reps=1)
+    fins = {}
+    for name in ("fini3", "passes"):
+        set_flatten(h, name)
+        f = forests[0].clone()
+        fins[name], _ = timed(lambda: h.finalize(f), reps=1)
+        del f
+    set_flatten(h, "passes")
+    h.finalize(forests[0])
+    set_flatten(h, "fini3")
+    t_fin = min(fins.values())
     torch.cuda.synchronize()
     ok = bool(torch.equal(forests[0], ref))
     t_rounds = sum(max(x["round_ms"] for x in v) for v in rounds.values())
     return {"merge_rounds": rounds, "final_flatten_ms": round(t_fin, 4),
+            "final_flatten_variants_ms": {k: round(v, 4) for k, v in fins.items()},
             "merge_total_ms": round(t_rounds + t_fin, 4), "labels_exact": ok,
             "projected_ms": round(max(t_rank) + t_rounds + t_fin, 4)}
 
 
+FLATTEN = {"fini3": dict(fini=3, flatten_passes=0), "fini1": dict(fini=1, flatten_passes=0),
+           "fini2": dict(fini=2, flatten_passes=0), "passes": dict(fini=3, flatten_passes=1)}
+
+
+def set_flatten(h, name):
+    for k, v in FLATTEN[name].items():
+        h.set_option(k, v)
+
+
 def encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank):
-    """Flatten + encode on every rank g > 0, one merge of all encodings into rank 0."""
-    encs, t_prep, pair_counts = [], [], []
+    """Every rank flattens its local forest (variants of ecl_cc_finalize timed: Fini3,
+    Fini1, Fini2, R23 passes + Fini3), ranks g > 0 encode; rank 0 merges all encodings in
+    one ecl_cc_merge_encoded call on its flattened forest and flattens once more."""
+    flat_ms = {}
+    for name in FLATTEN:
+        set_flatten(h, name)
+        per = []
+        for r in range(G):
+            f = forests[r].clone()
+            t_copy, _ = timed(lambda: f.copy_(forests[r]))
+            t, _ = timed(lambda: (f.copy_(forests[r]), h.finalize(f)))
+            per.append(round(max(t - t_copy, 0.0), 4))
+            del f
+        flat_ms[name] = per
+    best = min(flat_ms, key=lambda k: max(flat_ms[k]))
+    set_flatten(h, best)
+    flat = []
+    for r in range(G):
+        f = forests[r].clone()
+        h.finalize(f)
+        flat.append(f)
+    encs, t_enc, pair_counts = [], [], []
     for r in range(1, G):
         idx = nidx64[bounds[r]:bounds[r + 1] + 1]
         anchor = edist.row_anchor(idx, bounds[r])
         enc = h.encode_buffers(n)
-        f = forests[r].clone()
-
-        def prep():
-            f.copy_(forests[r])
-            h.finalize(f)
-            h.forest_encode(f, anchor, enc)
-        t_copy, _ = timed(lambda: f.copy_(forests[r]))
-        t, _ = timed(prep)
-        t_prep.append(max(t - t_copy, 0.0))
+        t, _ = timed(lambda: h.forest_encode(flat[r], anchor, enc))
+        t_enc.append(t)
         pair_counts.append(int(enc["meta"][0]))
         encs.append(enc)
-        del f
-    base = forests[0].clone()
+    base = flat[0].clone()
 
     def mrg():
-        forests[0].copy_(base)
-        h.merge_encoded(forests[0], encs)
-    copy_t, _ = timed(lambda: forests[0].copy_(base))
+        flat[0].copy_(base)
+        h.merge_encoded(flat[0], encs)
+    copy_t, _ = timed(lambda: flat[0].copy_(base))
     t_m, _ = timed(mrg)
     t_m = max(t_m - copy_t, 0.0)
-    forests[0].copy_(base)
-    h.merge_encoded(forests[0], encs)
-    t_fin, _ = timed(lambda: h.finalize(forests[0]), reps=1)
+    flat[0].copy_(base)
+    h.merge_encoded(flat[0], encs)
+    set_flatten(h, "fini3")
+    t_fin, _ = timed(lambda: h.finalize(flat[0]), reps=1)
     torch.cuda.synchronize()
-    ok = bool(torch.equal(forests[0], ref))
+    ok = bool(torch.equal(flat[0], ref))
     enc_bytes = sum(((n + 31) // 32) * 4 + 16 + 8 * c for c in pair_counts)
     xfer = enc_bytes / (args.link_gbs * 1e9) * 1e3
-    ready = max([t_rank[0]] + [t_rank[r] + t_prep[r - 1] for r in range(1, G)])
+    ready = max([t_rank[0] + flat_ms[best][0]] +
+                [t_rank[r] + flat_ms[best][r] + t_enc[r - 1] for r in range(1, G)])
     p2p = ready + max(t_m, xfer) + t_fin
     compact = ready + xfer + t_m + t_fin
-    return {"prep_ms": [round(x, 4) for x in t_prep], "pairs": pair_counts,
+    return {"flatten_ms": flat_ms, "flatten_used": best,
+            "encode_ms": [round(x, 4) for x in t_enc], "pairs": pair_counts,
             "encoded_bytes_total": enc_bytes, "merge_ms": round(t_m, 4),
             "transfer_ms_model": round(xfer, 4), "final_flatten_ms": round(t_fin, 4),
             "merge_total_p2p_ms": round(max(t_m, xfer) + t_fin, 4),
