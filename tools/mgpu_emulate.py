@@ -47,6 +47,23 @@ def timed(fn, reps=3):
     return best, out
 
 
+def depth_stats(parent):
+    """Mean / max depth (pointers to the root) of a forest, by pointer doubling."""
+    anc = parent.to(torch.int64)
+    ar = torch.arange(anc.numel(), device=anc.device)
+    dist = (anc != ar).to(torch.int64)
+    for _ in range(40):
+        nxt = anc[anc]
+        if torch.equal(nxt, anc):
+            break
+        dist = dist + dist[anc] * (anc != nxt)
+        anc = nxt
+    nonroot = parent.to(torch.int64) != ar
+    return {"mean_depth_nonroots": round(float(dist[nonroot].double().mean()), 3)
+            if bool(nonroot.any()) else 0.0, "max_depth": int(dist.max()),
+            "nonroots": int(nonroot.sum())}
+
+
 def tree_merge(h, forests, G, n, args, ref, t_rank):
     rounds = {}
     for (rd, send, recv) in edist.tree_schedule(G):
@@ -134,6 +151,11 @@ def encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank):
     copy_t, _ = timed(lambda: flat[0].copy_(base))
     t_m, _ = timed(mrg)
     t_m = max(t_m - copy_t, 0.0)
+    hs = ecl.Handle(0, stats=True)
+    f = base.clone()
+    hs.merge_encoded(f, encs)
+    merge_stats = hs.stats()
+    del f, hs
     flat[0].copy_(base)
     h.merge_encoded(flat[0], encs)
     set_flatten(h, "fini3")
@@ -146,7 +168,7 @@ def encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank):
                 [t_rank[r] + flat_ms[best][r] + t_enc[r - 1] for r in range(1, G)])
     p2p = ready + max(t_m, xfer) + t_fin
     compact = ready + xfer + t_m + t_fin
-    return {"flatten_ms": flat_ms, "flatten_used": best,
+    return {"flatten_ms": flat_ms, "flatten_used": best, "merge_stats": merge_stats,
             "encode_ms": [round(x, 4) for x in t_enc], "pairs": pair_counts,
             "encoded_bytes_total": enc_bytes, "merge_ms": round(t_m, 4),
             "transfer_ms_model": round(xfer, 4), "final_flatten_ms": round(t_fin, 4),
@@ -188,7 +210,10 @@ def main():
             t_rank.append(t)
             forests.append(par)
             del idx, lst
-        row = {"gpus": G, "rank_forest_ms": [round(x, 4) for x in t_rank]}
+        row = {"gpus": G, "rank_forest_ms": [round(x, 4) for x in t_rank],
+               "rank_entries": [int(nidx64[bounds[r + 1]] - nidx64[bounds[r]]) for r in range(G)],
+               "rank_rows": [bounds[r + 1] - bounds[r] for r in range(G)],
+               "rank_depth": [depth_stats(f) for f in forests] if G > 1 else None}
         if "tree" in args.merge and G > 1:
             tf = [f.clone() for f in forests]
             row["tree"] = tree_merge(h, tf, G, n, args, ref, t_rank)
