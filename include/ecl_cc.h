@@ -277,11 +277,22 @@ typedef enum {
                                      2 (default) only when a sample of the Init3
                                      forest is deep (meshes, road-like graphs).
                                      Labels are unchanged (R13).                       */
-    ECL_CC_OPT_FLATTEN_PASSES = 18 /* ecl_cc_finalize only: run R23's pointer-jumping
+    ECL_CC_OPT_FLATTEN_PASSES = 18, /* ecl_cc_finalize only: run R23's pointer-jumping
                                      passes before the finalize kernel: 0 (default) off,
                                      1 always, 2 when a depth probe finds the forest deep.
                                      For merged multi-GPU forests, whose former roots
                                      form long chains that Fini3 would walk per vertex. */
+    ECL_CC_OPT_FUSE_INIT = 19     /* Init3 folded into the hook kernels (R28):
+                                     the init kernel only bins rows by degree and writes
+                                     parent[v] = v; the kernel that owns a row's start
+                                     CASes parent[v] from v to the first smaller
+                                     neighbour (Init3's value) if v is still a root.
+                                     0 off (separate Init3 pass), 1 on, 2 (default) on
+                                     when m >= 16 n.  Applies with INIT 3 and STOP_AFTER
+                                     != 1 (the Init3 stage then uses the separate pass);
+                                     the R23 passes are skipped.  Labels unchanged (R13);
+                                     the worklists then hold every row of their degree
+                                     range, not only rows with a smaller neighbour.    */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

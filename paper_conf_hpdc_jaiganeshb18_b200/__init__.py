@@ -46,6 +46,7 @@ OPT = {
     "order": 16,
     "prejump": 17,
     "flatten_passes": 18,
+    "fuse_init": 19,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

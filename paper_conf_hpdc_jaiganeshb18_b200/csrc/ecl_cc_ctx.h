@@ -43,6 +43,7 @@ struct ecl_cc_ctx {
     cudaEvent_t done = nullptr;           // recorded at the end of every enqueueing call
     bool done_valid = false;
     int prejump = 2;                      // R23 pointer-doubling passes: 0 off, 1 on, 2 auto
+    int fuse_init = 2;                    // R28 lazy Init3: 0 off, 1 on, 2 auto (m >= 16n)
     int flatten_passes = 0;               // ecl_cc_finalize: R23 passes first (0 off,
                                           //   1 always, 2 if the depth probe finds it deep)
     int *fa = nullptr, *fb = nullptr;     // spanning-forest outputs of the current call

@@ -69,6 +69,12 @@ def test_algorithmic_bytes_partition_b_alg():
         for k in e:
             assert info[f"{k}_entries"] == e[k] and info[f"{k}_vertices"] == nv[k], (name, k)
         assert info["active"] == int((init3 != np.arange(g.n)).sum())
+        lz, li = bench.algorithmic_bytes(g, torch.from_numpy(init3), (16, 352), lazy=True)
+        assert sum(lz.values()) == sum(alg.values())
+        assert lz["init_bin"] == s_idx * (g.n + 1)          # R28: only nindex
+        deg = np.diff(nidx.astype(np.int64))
+        assert li["thread_entries"] == int(deg[deg <= 16].sum())
+        assert li["block_entries"] == int(deg[deg > 352].sum())
 
 
 def test_l2_probe_ceiling_uses_the_committed_measurement():

@@ -16,7 +16,8 @@ import paper_conf_hpdc_jaiganeshb18_b200 as ecl
 pytestmark = pytest.mark.gpu
 
 DEFAULTS = {"thresh_thread": 16, "thresh_warp": 352, "load_mode": 1, "ttas": 1, "init": 3,
-            "jump": 4, "fini": 3, "batch": 1, "filter": 2, "order": 2, "prejump": 2}
+            "jump": 4, "fini": 3, "batch": 1, "filter": 2, "order": 2, "prejump": 2,
+            "fuse_init": 2, "flatten_passes": 0}
 
 
 @pytest.fixture(scope="module")
@@ -174,9 +175,10 @@ def test_init3_stage(h, name):
 
 
 def test_worklist_sets(h):
-    """Bins (reading R2/R3): front = active with 16 < deg <= 352, back = deg > 352."""
+    """Bins (reading R2/R3): front = active with 16 < deg <= 352, back = deg > 352
+    (the separate Init3 pass; with R28 the bins hold every row of the degree range)."""
     g = gg.make_config("C4", seed=1, scale_down=4, device="cuda")
-    gpu_labels(h, g)
+    gpu_labels(h, g, fuse_init=0)
     front, back = h.worklist()
     nidx, nl = g.numpy()
     deg = np.diff(nidx.astype(np.int64))
@@ -185,6 +187,10 @@ def test_worklist_sets(h):
     eb = np.nonzero(active & (deg > 352))[0]
     assert np.array_equal(np.sort(front.cpu().numpy()), ef)
     assert np.array_equal(np.sort(back.cpu().numpy()), eb)
+    gpu_labels(h, g, fuse_init=1)                     # R28: degree-only bins
+    front, back = h.worklist()
+    assert np.array_equal(np.sort(front.cpu().numpy()), np.nonzero((deg > 16) & (deg <= 352))[0])
+    assert np.array_equal(np.sort(back.cpu().numpy()), np.nonzero(deg > 352)[0])
 
 
 def test_run_host_end_to_end(h):
@@ -231,18 +237,21 @@ def test_validate(h):
 
 def test_stats_identity():
     """-DECL_CC_STATS build: each successful hook CAS removes exactly one root, and
-    halving stores never create one, so #successful CAS == #Init3 roots - #CC (§8c)."""
+    halving stores never create one, so #successful CAS == #Init3 roots - #CC (§8c).
+    With R28 (Init3 folded into the hook kernels) the forest starts as n roots and the
+    Init CASes count too: #successful CAS == n - #CC."""
     with ecl.Handle(0, stats=True) as hs:
         assert hs.stats_enabled
         for name in ("C1", "C3", "C4"):
             g = gg.make_config(name, seed=1, scale_down=SMALL[name], device="cuda")
-            got = gpu_labels(hs, g)
-            st = hs.stats()
             nidx, nl = g.numpy()
             expect, ncc = oracle.bfs(nidx, nl)
-            assert np.array_equal(got, expect)
             roots = int((oracle.init3(nidx, nl) == np.arange(g.n)).sum())
-            assert st["cas_success"] == roots - ncc, (name, st, roots, ncc)
+            for fuse, start in ((0, roots), (1, g.n)):
+                got = gpu_labels(hs, g, fuse_init=fuse)
+                st = hs.stats()
+                assert np.array_equal(got, expect)
+                assert st["cas_success"] == start - ncc, (name, fuse, st, start, ncc)
 
 
 def test_pre_finalize_forest_invariant(h):
@@ -578,3 +587,54 @@ def test_path_length_counters():
             assert st["find_walks"] <= st["path_len_sum"] <= st["path_len_max"] * st["find_walks"]
             res[jump] = st["path_len_sum"] / st["find_walks"]
         assert res[3] >= res[4]
+
+
+# ---------------------------------------------------------------------------------------
+# R28 lazy Init3 (Init3 folded into the hook kernels): forced on and off everywhere
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("fuse", [0, 1])
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("seed", [1, 2])
+def test_fuse_init_configs(h, name, fuse, seed):
+    g = gg.make_config(name, seed=seed + 40, scale_down=SMALL[name], device="cuda")
+    assert_parity(h, g, fuse_init=fuse)
+    assert_parity(h, gg.shuffle_rows(g, seed=seed), fuse_init=fuse, order=0)
+
+
+@pytest.mark.parametrize("g", hand_graphs(), ids=lambda g: g.name)
+def test_fuse_init_hand_built(h, g):
+    assert_parity(h, g, fuse_init=1)
+    assert_forest(h, g, fuse_init=1)
+
+
+@pytest.mark.parametrize("opts", [dict(filter=1), dict(filter=0), dict(grid_blocks=3),
+                                  dict(load_mode=0), dict(batch=0), dict(jump=2),
+                                  dict(thresh_thread=4, thresh_warp=8), dict(order=1)],
+                         ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
+def test_fuse_init_options(h, opts):
+    g = gg.make_config("C5", seed=3, scale_down=9, device="cuda")
+    assert_parity(h, g, fuse_init=1, **opts)
+    assert_forest(h, gg.make_config("C4", seed=3, scale_down=8, device="cuda"), fuse_init=1,
+                  **opts)
+
+
+@pytest.mark.parametrize("G", [2, 4])
+def test_fuse_init_multi_gpu(h, G):
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config("C5", seed=5, scale_down=10, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64, G)
+    h.set_option("fuse_init", 1)
+    try:
+        forests = []
+        for r in range(G):
+            idx, lst = dist.slice_rows(nindex64, g.nlist, bounds[r], bounds[r + 1])
+            forests.append(h.run_rows(g.n, bounds[r], bounds[r + 1], idx, lst, flatten=False))
+        for (_, send, recv) in dist.tree_schedule(G):
+            h.merge(forests[recv], forests[send])
+        h.finalize(forests[0])
+        torch.cuda.synchronize()
+    finally:
+        h.set_option("fuse_init", 2)
+    assert np.array_equal(forests[0].cpu().numpy(), expect)

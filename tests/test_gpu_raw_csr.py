@@ -89,6 +89,7 @@ def labels(h, g, index_dtype=None, **opts):
     finally:
         h.set_option("order", 2)
         h.set_option("prejump", 2)
+        h.set_option("fuse_init", 2)
     return out.cpu().numpy()
 
 
@@ -109,9 +110,10 @@ def has_loops_and_dups(g):
 @pytest.mark.parametrize("g", hand_raw_graphs(), ids=lambda g: g.name)
 @pytest.mark.parametrize("order", [0, 2])
 @pytest.mark.parametrize("index_dtype", [torch.int32, torch.int64], ids=["i32", "i64"])
-def test_hand_raw(h, g, order, index_dtype):
+@pytest.mark.parametrize("fuse", [0, 1])
+def test_hand_raw(h, g, order, index_dtype, fuse):
     exp = expected(g)
-    got = labels(h, g, index_dtype=index_dtype, order=order)
+    got = labels(h, g, index_dtype=index_dtype, order=order, fuse_init=fuse)
     assert np.array_equal(got, exp), g.name
 
 
@@ -125,6 +127,8 @@ def test_configs_with_loops_dups(h, name, order):
     assert np.array_equal(exp, expected(clean))          # "same as cleaned"
     assert np.array_equal(labels(h, g, order=order), exp)
     assert np.array_equal(labels(h, g, index_dtype=torch.int64, order=order), exp)
+    for fuse in (0, 1):
+        assert np.array_equal(labels(h, g, order=order, fuse_init=fuse), exp)
 
 
 @pytest.mark.parametrize("name", ["C4", "C5"])
@@ -148,15 +152,15 @@ def test_hand_raw_init_stage(h, g):
     assert np.array_equal(got, oracle.init3(*g.numpy()))
 
 
-def _forest(h, g, index_dtype=None, order=2):
+def _forest(h, g, index_dtype=None, order=2, fuse=2):
     g = g.to("cuda")
     nindex = g.nindex if index_dtype is None else g.nindex.to(index_dtype)
-    h.set_option("order", order)
+    h.set_option("order", order).set_option("fuse_init", fuse)
     try:
         lab, ta, tb = h.spanning_forest(nindex, g.nlist)
         torch.cuda.synchronize()
     finally:
-        h.set_option("order", 2)
+        h.set_option("order", 2).set_option("fuse_init", 2)
     nidx, nl = g.numpy()
     exp = expected(g)
     assert np.array_equal(lab.cpu().numpy(), exp)
@@ -168,8 +172,9 @@ def _forest(h, g, index_dtype=None, order=2):
 
 @pytest.mark.parametrize("g", hand_raw_graphs(), ids=lambda g: g.name)
 @pytest.mark.parametrize("order", [0, 2])
-def test_forest_hand_raw(h, g, order):
-    _forest(h, g, order=order)
+@pytest.mark.parametrize("fuse", [0, 1])
+def test_forest_hand_raw(h, g, order, fuse):
+    _forest(h, g, order=order, fuse=fuse)
 
 
 @pytest.mark.parametrize("name", ["C2", "C4", "C5"])
@@ -178,3 +183,4 @@ def test_forest_configs_with_loops_dups(h, name):
                                             device="cuda"), seed=8)
     _forest(h, g, order=0)
     _forest(h, g, index_dtype=torch.int64, order=2)
+    _forest(h, g, order=2, fuse=1)
