@@ -123,9 +123,10 @@ def build_graph(name: str, seed: int, device, scale_down: int = 0):
     return g, time.time() - t0
 
 
-def lazy_init_used(g) -> bool:
-    """The library's default choice of R28 (ECL_CC_OPT_FUSE_INIT auto): m >= 16 n."""
-    return g.m >= 16 * g.n
+def lazy_init_used(g) -> int:
+    """The library's default R28 mode (ECL_CC_OPT_FUSE_INIT auto): 3 (rows above the
+    thread bin get their Init3 parent in hook_range) when m >= 16 n, else 0."""
+    return 3 if g.m >= 16 * g.n else 0
 
 
 def algorithmic_bytes(g, parent_init, hw, lazy=False):
@@ -139,8 +140,9 @@ def algorithmic_bytes(g, parent_init, hw, lazy=False):
       hook_warp    4 B per entry of the worklist-front rows (17..352)
       hook_block   4 B per entry of the worklist-back rows (> 352)
       finalize     4 B per label written
-    With R28 (lazy: Init3 folded into the hook kernels) init_bin reads only nindex and the
-    hook kernels read every entry of the rows of their degree range.
+    With R28 (lazy: Init3 folded into the hook kernels) the range kernels read every entry
+    of the rows of their degree range; with lazy == 1 so does hook_thread and init_bin
+    reads only nindex.
     parent_init = Init3 parents (a stop_after=1 run) on the device."""
     n, m = g.n, g.m
     s_idx = g.nindex.element_size()
@@ -163,11 +165,12 @@ def algorithmic_bytes(g, parent_init, hw, lazy=False):
         x = g.nlist[starts[sel] + j].to(torch.int64)
         other[sel] = other[sel] | ((x < v[sel]) & (x != par[sel]))
     tw = thr & (~small | other)
-    if lazy:
-        nz = deg > 0
-        thr, tw = nz & (deg <= t1), nz & (deg <= t1)
+    if lazy:            # R28: rows above the thread bin are streamed whether active or not
         fr = (deg > t1) & (deg <= t2)
         bk = deg > t2
+    if lazy == 1:       # ... and every thread-bin row too (init reads no row)
+        nz = deg > 0
+        thr, tw = nz & (deg <= t1), nz & (deg <= t1)
     e_thr, e_fr, e_bk = (int(deg[x].sum()) for x in (tw, fr, bk))
     b = {
         "init_bin": s_idx * (n + 1) + 4 * (m - e_thr - e_fr - e_bk),
@@ -384,6 +387,8 @@ def main():
     ap.add_argument("--load-mode", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--chunks", type=int, default=4, help="tree merge: chunks per round")
+    ap.add_argument("--calibrate", type=int, default=1,
+                    help="N > 1: re-partition once from measured local-forest times")
     ap.add_argument("--merge", default="p2p", choices=["p2p", "compact", "tree"],
                     help="N > 1: forest merge (dist.EncodedMerge p2p / compact, or the "
                          "binomial tree of full forests)")
@@ -424,7 +429,8 @@ def main():
         h.set_option("stop_after", 0)
         lazy = lazy_init_used(g)
         alg, info = algorithmic_bytes(g, labels, (16, 352), lazy=lazy)
-        info["init"] = "R28 lazy Init3 in the hook kernels" if lazy else "separate Init3 pass"
+        info["init"] = {0: "separate Init3 pass", 1: "R28: Init3 in the hook kernels",
+                        3: "R28: Init3 of rows > 16 entries in hook_range"}[lazy]
 
     if world == 1:
         step = lambda: h.run(g.nindex, g.nlist, out=labels)  # noqa: E731
@@ -432,8 +438,28 @@ def main():
         # rows split by estimated work (probed entries + a streaming share); every rank
         # keeps ONLY its slice resident (the full graph is built once to cut it, outside
         # the timed region, and released)
-        bounds = edist.partition_rows(g.nindex, world,
-                                      weights=edist.row_weights(g.nindex, g.nlist))
+        wts = edist.row_weights(g.nindex, g.nlist)
+        bounds = edist.partition_rows(g.nindex, world, weights=wts)
+        calib = None
+        if args.calibrate:
+            # one measured local forest per rank re-weights the rows (setup, untimed)
+            lo, hi = bounds[rank], bounds[rank + 1]
+            i0, l0 = edist.slice_rows(g.nindex, g.nlist, lo, hi)
+            ts = []
+            for _ in range(3):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                h.run_rows(n, lo, hi, i0, l0, parent=labels, flatten=False)
+                e1.record(stream)
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            t = torch.tensor([min(ts)], dtype=torch.float64, device=dev)
+            allt = [torch.zeros_like(t) for _ in range(world)]
+            tdist.all_gather(allt, t)
+            calib = [round(float(x.item()), 4) for x in allt]
+            bounds = edist.partition_rows(g.nindex, world,
+                                          weights=edist.rebalance_weights(wts, bounds, calib))
+            del i0, l0
         lo, hi = bounds[rank], bounds[rank + 1]
         idx_r, lst_r = edist.slice_rows(g.nindex, g.nlist, lo, hi)
         idx_r, lst_r = idx_r.clone(), lst_r.clone()
@@ -628,7 +654,9 @@ def main():
                    "parallelism": f"rows{world}" if world > 1 else "single",
                    "load_mode": args.load_mode, "gen_s": round(gen_s, 1), **info,
                    **({"rank0_rows": [lo, hi], "rank0_entries": slice_entries,
-                       "merge": args.merge, "merge_chunks": args.chunks}
+                       "merge": args.merge, "merge_chunks": args.chunks,
+                       "partition": "row_weights" + (" + calibrated" if calib else ""),
+                       "calibration_forest_ms": calib}
                       if world > 1 else {})},
         "gpu_launches": launches_per_step(world, rank, args.chunks, args.merge) * args.steps,
         "clocks": clk.summary(),

@@ -287,8 +287,11 @@ typedef enum {
                                      parent[v] = v; the kernel that owns a row's start
                                      CASes parent[v] from v to the first smaller
                                      neighbour (Init3's value) if v is still a root.
-                                     0 off (separate Init3 pass), 1 on, 2 (default) on
-                                     when m >= 16 n.  Applies with INIT 3 and STOP_AFTER
+                                     0 off (separate Init3 pass), 1 every row, 3 only
+                                     the rows above the thread bin (the init kernel
+                                     still sets the thread-bin rows' Init3 parents),
+                                     2 (default) = 3 when m >= 16 n, else 0.
+                                     Applies with INIT 3 and STOP_AFTER
                                      != 1 (the Init3 stage then uses the separate pass);
                                      the R23 passes are skipped.  Labels unchanged (R13);
                                      the worklists then hold every row of their degree

@@ -105,10 +105,11 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     // R28: Init3 folded into the hook kernels (the separate pass over every row start is
     // then a degree-only binning pass); auto = graphs with long rows (m >= 16 n), where
     // that pass reads one sector per row for a few bytes
-    const bool lazy = h->init_mode == 3 && h->stop_after != 1 &&
-                      (h->fuse_init == 1 || (h->fuse_init == 2 && m >= 16LL * nrows));
-    p.lazy = lazy ? 1 : 0;
-    p.init_mode = lazy ? 1 : h->init_mode;   // the binning pass: parent[v] = v, bins by degree
+    const int fuse = h->fuse_init == 2 ? (m >= 16LL * nrows ? 3 : 0) : h->fuse_init;
+    const bool lazy = h->init_mode == 3 && h->stop_after != 1 && fuse != 0;
+    p.lazy = !lazy ? 0 : fuse == 1 ? 1 : 2;
+    // every row lazy: the binning pass is Init1's (parent[v] = v, bins by degree)
+    p.init_mode = p.lazy == 1 ? 1 : h->init_mode;
     p.jump = h->jump;
     p.batch = h->batch;
     p.anchor = h->cnt + 10;
@@ -151,7 +152,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         auto k = init_bin_kernel<idx_t>;
         k<<<grid_for(h, (const void *)k, ((long long)nrows + kInitPerThread - 1) / kInitPerThread), kBlock, 0, s>>>(p);
     }
-    if (h->prejump != 0 && h->stop_after != 1 && nrows > 0 && !lazy) {
+    if (h->prejump != 0 && h->stop_after != 1 && nrows > 0 && p.lazy != 1) {
         // R23: depth probe, then the passes (cooperative launch guarantees the
         // co-residency their grid barrier needs); both are no-ops on shallow forests
         int *ctl = (int *)(h->cnt + 4);
@@ -777,7 +778,7 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         h->prejump = (int)value;
         break;
     case ECL_CC_OPT_FUSE_INIT:
-        if (value < 0 || value > 2) return fail_arg(h, "fuse_init must be 0, 1 or 2");
+        if (value < 0 || value > 3) return fail_arg(h, "fuse_init must be 0..3");
         h->fuse_init = (int)value;
         break;
     case ECL_CC_OPT_FLATTEN_PASSES:

@@ -70,6 +70,24 @@ def partition_rows(nindex: torch.Tensor, world: int,
     return bounds
 
 
+def rebalance_weights(weights: torch.Tensor, bounds: List[int], rank_ms) -> torch.Tensor:
+    """Per-row weights rescaled by each rank's MEASURED cost per weight unit (one untimed
+    step of the current partition), for a second partition_rows call.  The static
+    weights miss costs that depend on where the rows sit in the ID order: the owner of the
+    highest IDs finds its rows' Init3 parents outside its range (identity roots)
+    and does more hooking per probed entry."""
+    w = weights.to(torch.float64).cpu().clone()
+    for r in range(len(bounds) - 1):
+        lo, hi = bounds[r], bounds[r + 1]
+        tot = float(w[lo:hi].sum())
+        if tot > 0 and rank_ms[r] > 0:
+            w[lo:hi] *= float(rank_ms[r]) / tot
+    total = float(w.sum())
+    if total <= 0:
+        return weights
+    return (w * (2.0 ** 40 / total)).round().to(torch.int64)
+
+
 def slice_rows(nindex: torch.Tensor, nlist: torch.Tensor, lo: int, hi: int):
     """CSR slice of rows [lo, hi): int64 offsets rebased to 0, and the adjacency view."""
     nindex = nindex.to(torch.int64)

@@ -69,12 +69,16 @@ def test_algorithmic_bytes_partition_b_alg():
         for k in e:
             assert info[f"{k}_entries"] == e[k] and info[f"{k}_vertices"] == nv[k], (name, k)
         assert info["active"] == int((init3 != np.arange(g.n)).sum())
-        lz, li = bench.algorithmic_bytes(g, torch.from_numpy(init3), (16, 352), lazy=True)
+        lz, li = bench.algorithmic_bytes(g, torch.from_numpy(init3), (16, 352), lazy=1)
         assert sum(lz.values()) == sum(alg.values())
         assert lz["init_bin"] == s_idx * (g.n + 1)          # R28: only nindex
         deg = np.diff(nidx.astype(np.int64))
         assert li["thread_entries"] == int(deg[deg <= 16].sum())
         assert li["block_entries"] == int(deg[deg > 352].sum())
+        l3, i3 = bench.algorithmic_bytes(g, torch.from_numpy(init3), (16, 352), lazy=3)
+        assert sum(l3.values()) == sum(alg.values())
+        assert i3["thread_entries"] == info["thread_entries"]
+        assert i3["warp_entries"] == int(deg[(deg > 16) & (deg <= 352)].sum())
 
 
 def test_l2_probe_ceiling_uses_the_committed_measurement():

@@ -155,3 +155,17 @@ def test_forest_merge_gloo(world, chunks, broadcast):
             assert np.array_equal(results[r], expect)
         else:
             assert results[r] is None
+
+
+def test_rebalance_weights_moves_rows_off_slow_ranks():
+    """A rank measured twice as slow per weight unit gets fewer rows after rebalancing;
+    equal measured times leave the partition (nearly) unchanged."""
+    w = torch.ones(1000, dtype=torch.int64) * 4
+    b = edist.partition_rows(torch.arange(1001), 4, weights=w)
+    assert b == [0, 250, 500, 750, 1000]
+    nb = edist.partition_rows(torch.arange(1001), 4,
+                              weights=edist.rebalance_weights(w, b, [1.0, 1.0, 1.0, 2.0]))
+    assert nb[0] == 0 and nb[-1] == 1000 and nb[4] - nb[3] < 250 and nb[1] > 250
+    same = edist.partition_rows(torch.arange(1001), 4,
+                                weights=edist.rebalance_weights(w, b, [3.0, 3.0, 3.0, 3.0]))
+    assert all(abs(x - y) <= 1 for x, y in zip(same, b))

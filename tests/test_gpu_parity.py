@@ -592,7 +592,7 @@ def test_path_length_counters():
 # ---------------------------------------------------------------------------------------
 # R28 lazy Init3 (Init3 folded into the hook kernels): forced on and off everywhere
 # ---------------------------------------------------------------------------------------
-@pytest.mark.parametrize("fuse", [0, 1])
+@pytest.mark.parametrize("fuse", [0, 1, 3])
 @pytest.mark.parametrize("name", list(SMALL))
 @pytest.mark.parametrize("seed", [1, 2])
 def test_fuse_init_configs(h, name, fuse, seed):
@@ -603,8 +603,9 @@ def test_fuse_init_configs(h, name, fuse, seed):
 
 @pytest.mark.parametrize("g", hand_graphs(), ids=lambda g: g.name)
 def test_fuse_init_hand_built(h, g):
-    assert_parity(h, g, fuse_init=1)
-    assert_forest(h, g, fuse_init=1)
+    for fuse in (1, 3):
+        assert_parity(h, g, fuse_init=fuse)
+        assert_forest(h, g, fuse_init=fuse)
 
 
 @pytest.mark.parametrize("opts", [dict(filter=1), dict(filter=0), dict(grid_blocks=3),
@@ -613,9 +614,10 @@ def test_fuse_init_hand_built(h, g):
                          ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
 def test_fuse_init_options(h, opts):
     g = gg.make_config("C5", seed=3, scale_down=9, device="cuda")
-    assert_parity(h, g, fuse_init=1, **opts)
-    assert_forest(h, gg.make_config("C4", seed=3, scale_down=8, device="cuda"), fuse_init=1,
-                  **opts)
+    for fuse in (1, 3):
+        assert_parity(h, g, fuse_init=fuse, **opts)
+        assert_forest(h, gg.make_config("C4", seed=3, scale_down=8, device="cuda"),
+                      fuse_init=fuse, **opts)
 
 
 @pytest.mark.parametrize("G", [2, 4])

@@ -22,10 +22,14 @@ import torch  # noqa: E402
 import graphgen as gg  # noqa: E402
 import paper_conf_hpdc_jaiganeshb18_b200 as ecl  # noqa: E402
 
+# Jump1-3 exist only on the plain path (one find + hook per edge, no R19/R22 batching),
+# so "Jump4_plain" (batch 0) is their like-for-like baseline: relative_to_jump4_plain
 VARIANTS = [("base", {}), ("Init1", {"init": 1}), ("Init2", {"init": 2}),
+            ("Jump4_plain", {"batch": 0}),
             ("Jump1", {"jump": 1}), ("Jump2", {"jump": 2}), ("Jump3", {"jump": 3}),
-            ("Fini1", {"fini": 1}), ("Fini2", {"fini": 2})]
-DEF = {"init": 3, "jump": 4, "fini": 3}
+            ("Fini1", {"fini": 1}), ("Fini2", {"fini": 2}),
+            ("separate_Init3_pass", {"fuse_init": 0})]
+DEF = {"init": 3, "jump": 4, "fini": 3, "batch": 1, "fuse_init": 2}
 L2 = 126 << 20
 
 
@@ -83,7 +87,13 @@ def main():
                          flush)
             assert torch.equal(out, ref), (c, name)
             row["relative_runtime"][name] = round(t / base, 3)
+            row.setdefault("ms", {})[name] = round(t, 4)
             row["paths"][name] = paths(hs, g, opts)
+        jp = row.get("ms", {}).get("Jump4_plain")
+        if jp:
+            row["relative_to_jump4_plain"] = {k: round(row["ms"][k] / jp, 3)
+                                              for k in ("Jump1", "Jump2", "Jump3")
+                                              if k in row["ms"]}
         print(json.dumps(row), flush=True)
         del g, flush
         torch.cuda.empty_cache()

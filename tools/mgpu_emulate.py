@@ -186,6 +186,8 @@ def main():
     ap.add_argument("--even", action="store_true")
     ap.add_argument("--order", type=int, default=2, help="ECL_CC_OPT_ORDER of every run")
     ap.add_argument("--merge", default="tree,encoded")
+    ap.add_argument("--calibrate", type=int, default=1,
+                    help="re-partition once from the measured local-forest times")
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=1, device="cuda")
     n, m = g.n, g.m
@@ -210,7 +212,25 @@ def main():
             t_rank.append(t)
             forests.append(par)
             del idx, lst
+        if args.calibrate and G > 1 and wts is not None:
+            # one measured step re-weights the rows (dist.rebalance_weights), then the
+            # local forests are rebuilt on the new partition
+            t_first = list(t_rank)
+            bounds = edist.partition_rows(nidx64.cpu(), G, weights=edist.rebalance_weights(
+                wts, bounds, t_rank))
+            del forests
+            forests, t_rank = [], []
+            for r in range(G):
+                lo, hi = bounds[r], bounds[r + 1]
+                idx, lst = edist.slice_rows(nidx64, g.nlist, lo, hi)
+                par = torch.empty(n, dtype=torch.int32, device="cuda")
+                t, _ = timed(lambda: h.run_rows(n, lo, hi, idx, lst, parent=par, flatten=False))
+                t_rank.append(t)
+                forests.append(par)
+                del idx, lst
         row = {"gpus": G, "rank_forest_ms": [round(x, 4) for x in t_rank],
+               "rank_forest_ms_before_calibration":
+                   [round(x, 4) for x in t_first] if args.calibrate and G > 1 else None,
                "rank_entries": [int(nidx64[bounds[r + 1]] - nidx64[bounds[r]]) for r in range(G)],
                "rank_rows": [bounds[r + 1] - bounds[r] for r in range(G)],
                "rank_depth": [depth_stats(f) for f in forests] if G > 1 else None}
