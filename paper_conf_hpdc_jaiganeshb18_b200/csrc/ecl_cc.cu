@@ -26,6 +26,10 @@ constexpr int kNumStats = 16;
 #define ECL_FAST_FINI 1
 #endif
 constexpr bool kFastFini = ECL_FAST_FINI != 0;   // Fini3 via finalize3_kernel
+#ifndef ECL_INIT_BRANGE
+#define ECL_INIT_BRANGE 1
+#endif
+constexpr bool kInitBlockRange = ECL_INIT_BRANGE != 0;   // init_bin: block-range mode
 
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
 
@@ -63,12 +67,21 @@ ecl_cc_status ensure_scratch(ecl_cc_handle h, int need, cudaStream_t s)
     if (h->wl) CK(cudaFreeAsync(h->wl, s), "cudaFreeAsync(wl)");
     if (h->ub) CK(cudaFreeAsync(h->ub, s), "cudaFreeAsync(ub)");
     if (h->tbits) CK(cudaFreeAsync(h->tbits, s), "cudaFreeAsync(tbits)");
+    if (h->scr) CK(cudaFreeAsync(h->scr, s), "cudaFreeAsync(scr)");
+    if (h->scru) CK(cudaFreeAsync(h->scru, s), "cudaFreeAsync(scru)");
     h->wl = nullptr;
     h->ub = nullptr;
     h->tbits = nullptr;
+    h->scr = nullptr;
+    h->scru = nullptr;
     h->cap = 0;
     CK(cudaMallocAsync((void **)&h->wl, sizeof(int) * (size_t)need, s), "cudaMallocAsync(wl)");
     CK(cudaMallocAsync((void **)&h->ub, sizeof(unsigned) * (size_t)need, s), "cudaMallocAsync(ub)");
+    if (kInitBlockRange) {
+        CK(cudaMallocAsync((void **)&h->scr, sizeof(int) * (size_t)need, s), "cudaMallocAsync(scr)");
+        CK(cudaMallocAsync((void **)&h->scru, sizeof(unsigned) * (size_t)need, s),
+           "cudaMallocAsync(scru)");
+    }
     CK(cudaMallocAsync((void **)&h->tbits, sizeof(unsigned) * (((size_t)need + 31) / 32), s),
        "cudaMallocAsync(tbits)");
     h->cap = need;
@@ -150,7 +163,20 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     }
     {
         auto k = init_bin_kernel<idx_t>;
-        k<<<grid_for(h, (const void *)k, ((long long)nrows + kInitPerThread - 1) / kInitPerThread), kBlock, 0, s>>>(p);
+        const int grid = grid_for(h, (const void *)k,
+                                  ((long long)nrows + kInitPerThread - 1) / kInitPerThread);
+        p.scr = nullptr;
+        p.scru = nullptr;
+        p.rows_per_block = 0;
+        if (kInitBlockRange && h->scr) {
+            // each block owns a contiguous range of whole chunks (one worklist reservation
+            // per block instead of one per chunk)
+            const long long chunks = ((long long)nrows + kInitChunk - 1) / kInitChunk;
+            p.scr = h->scr;
+            p.scru = h->scru;
+            p.rows_per_block = (int)(((chunks + grid - 1) / grid) * kInitChunk);
+        }
+        k<<<grid, kBlock, 0, s>>>(p);
     }
     if (h->prejump != 0 && h->stop_after != 1 && nrows > 0 && p.lazy != 1) {
         // R23: depth probe, then the passes (cooperative launch guarantees the
@@ -357,7 +383,7 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
         cudaStream_t s = h->side;
         if (h->done_valid) cudaStreamWaitEvent(s, h->done, 0);
         void *bufs[] = {h->wl, h->ub, h->tbits, h->cnt, h->flags, h->e2e_index, h->e2e_list,
-                        h->e2e_labels, h->gbits, h->csr_tmp};
+                        h->e2e_labels, h->gbits, h->csr_tmp, h->scr, h->scru};
         for (void *b : bufs)
             if (b) cudaFreeAsync(b, s);
         cudaStreamSynchronize(s);

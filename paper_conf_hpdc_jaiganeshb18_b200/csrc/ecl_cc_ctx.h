@@ -16,6 +16,8 @@ struct ecl_cc_ctx {
     int *wl = nullptr;
     unsigned *ub = nullptr;
     unsigned *tbits = nullptr;            // R24 thread-bin work bitmap (one bit per row)
+    int *scr = nullptr;                   // init_bin's per-block worklist staging (vertex,
+    unsigned *scru = nullptr;             //   block-local unit base), cap entries each
     int cap = 0;
     unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [8..9] int
                                           // scheduling counters, [10] R21 anchor,
