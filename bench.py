@@ -123,12 +123,6 @@ def build_graph(name: str, seed: int, device, scale_down: int = 0):
     return g, time.time() - t0
 
 
-def lazy_init_used(g) -> int:
-    """The library's default R28 mode (ECL_CC_OPT_FUSE_INIT auto): 3 (rows above the
-    thread bin get their Init3 parent in hook_range) when m >= 16 n, else 0."""
-    return 3 if g.m >= 16 * g.n else 0
-
-
 def algorithmic_bytes(g, parent_init, hw, lazy=False):
     """Per-kernel split of B_alg = S_idx(n+1) + 4m + 4n: every
     byte of B_alg is charged to exactly ONE kernel, so the parts sum to B_alg.
@@ -140,9 +134,8 @@ def algorithmic_bytes(g, parent_init, hw, lazy=False):
       hook_warp    4 B per entry of the worklist-front rows (17..352)
       hook_block   4 B per entry of the worklist-back rows (> 352)
       finalize     4 B per label written
-    With R28 (lazy: Init3 folded into the hook kernels) the range kernels read every entry
-    of the rows of their degree range; with lazy == 1 so does hook_thread and init_bin
-    reads only nindex.
+    With R28 (lazy: Init3 folded into the hook kernels) init_bin reads only nindex and the
+    hook kernels read every entry of the rows of their degree range.
     parent_init = Init3 parents (a stop_after=1 run) on the device."""
     n, m = g.n, g.m
     s_idx = g.nindex.element_size()
@@ -165,12 +158,11 @@ def algorithmic_bytes(g, parent_init, hw, lazy=False):
         x = g.nlist[starts[sel] + j].to(torch.int64)
         other[sel] = other[sel] | ((x < v[sel]) & (x != par[sel]))
     tw = thr & (~small | other)
-    if lazy:            # R28: rows above the thread bin are streamed whether active or not
-        fr = (deg > t1) & (deg <= t2)
-        bk = deg > t2
-    if lazy == 1:       # ... and every thread-bin row too (init reads no row)
+    if lazy:            # R28: every non-empty row is streamed by the kernel of its bin
         nz = deg > 0
         thr, tw = nz & (deg <= t1), nz & (deg <= t1)
+        fr = (deg > t1) & (deg <= t2)
+        bk = deg > t2
     e_thr, e_fr, e_bk = (int(deg[x].sum()) for x in (tw, fr, bk))
     b = {
         "init_bin": s_idx * (n + 1) + 4 * (m - e_thr - e_fr - e_bk),
@@ -359,15 +351,16 @@ def check_world(args) -> None:
         sys.exit(2)
 
 
-def launches_per_step(world: int, rank: int, chunks: int, merge: str) -> int:
+def launches_per_step(world: int, rank: int, chunks: int, merge: str, probe: int = 0) -> int:
     """Our kernels per step on `rank`: init_bin, depth_probe, prejump (exits at once on
-    shallow forests), hook_thread, hook_range x2, finalize; with G ranks: identity_outside
+    shallow forests), hook_thread, hook_range x2, finalize (+ `probe`: R28's locality
+    probe, launched when m < 16n); with G ranks: identity_outside
     instead of finalize in run_rows, then for the tree merge one merge_hook per received
     chunk and rank 0's finalize; for the encoded merges a flatten (R23 depth probe +
     passes + finalize) and encode on every rank g > 0, and on rank 0 a flatten,
     merge_bits + merge_pairs, and a flatten."""
     if world == 1:
-        return 7
+        return 7 + probe
     from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
     if merge != "tree":
         fl = 3 if edist.EncodedMerge.FLATTEN.get("flatten_passes") else 1
@@ -424,13 +417,16 @@ def main():
     # ---- algorithmic-bytes bookkeeping (outside the timed region; N=1 path) ----
     alg, info = {}, {}
     if world == 1:
+        h.run(g.nindex, g.nlist, out=labels)
+        run_info = h.run_info()                 # the library's own R28 / R23 decisions
+        lazy = 1 if run_info["lazy_init3"] else 0
         h.set_option("stop_after", 1)
         h.run(g.nindex, g.nlist, out=labels)
         h.set_option("stop_after", 0)
-        lazy = lazy_init_used(g)
         alg, info = algorithmic_bytes(g, labels, (16, 352), lazy=lazy)
-        info["init"] = {0: "separate Init3 pass", 1: "R28: Init3 in the hook kernels",
-                        3: "R28: Init3 of rows > 16 entries in hook_range"}[lazy]
+        info["init"] = "R28: Init3 in the hook kernels" if lazy else "separate Init3 pass"
+        info["r23_passes"] = run_info["deep_forest_passes"]
+        info["r21_filter"] = run_info["filter"]
 
     if world == 1:
         step = lambda: h.run(g.nindex, g.nlist, out=labels)  # noqa: E731
@@ -658,7 +654,8 @@ def main():
                        "partition": "row_weights" + (" + calibrated" if calib else ""),
                        "calibration_forest_ms": calib}
                       if world > 1 else {})},
-        "gpu_launches": launches_per_step(world, rank, args.chunks, args.merge) * args.steps,
+        "gpu_launches": launches_per_step(world, rank, args.chunks, args.merge,
+                                          probe=int(m < 16 * n)) * args.steps,
         "clocks": clk.summary(),
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},

@@ -287,11 +287,14 @@ typedef enum {
                                      parent[v] = v; the kernel that owns a row's start
                                      CASes parent[v] from v to the first smaller
                                      neighbour (Init3's value) if v is still a root.
-                                     0 off (separate Init3 pass), 1 every row, 3 only
-                                     the rows above the thread bin (the init kernel
-                                     still sets the thread-bin rows' Init3 parents),
-                                     2 (default) = 3 when m >= 16 n, else 0.
-                                     Applies with INIT 3 and STOP_AFTER
+                                     0 off (separate Init3 pass), 1 on, 2 (default)
+                                     auto: off when m >= 16 n, else decided on the
+                                     device by a one-block probe of 256 rows (on when
+                                     their first smaller neighbours are mostly far
+                                     from the row's ID, i.e. random vertex IDs; off
+                                     for meshes / road-like graphs, whose Init3 chains
+                                     the R23 passes shorten).  ecl_cc_get_run_info
+                                     reports the decision.  Applies with INIT 3 and STOP_AFTER
                                      != 1 (the Init3 stage then uses the separate pass);
                                      the R23 passes are skipped.  Labels unchanged (R13);
                                      the worklists then hold every row of their degree
@@ -321,6 +324,19 @@ ECL_CC_API ecl_cc_status ecl_cc_get_stats(ecl_cc_handle h, int64_t out[4]);
  * nor edges the R21/R22 probe settles without a walk): [13] sum of lengths, [14] walks,
  * [15] maximum length. */
 ECL_CC_API ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int count);
+
+/* Debug: what the most recent run decided (synchronises it); count <= 4:
+ * [0] 1 if Init3 ran inside the hook kernels (R28), [1] 1 if the R23 depth probe found a
+ * deep forest (the pointer-jumping passes ran), [2] 1 if the R21 bitmap filter was on,
+ * [3] the R21 anchor vertex (-1 if none). */
+ECL_CC_API ecl_cc_status ecl_cc_get_run_info(ecl_cc_handle h, int64_t *out, int count);
+
+/* Debug: the handle's R21 anchor-tree membership bitmap (R21) as left by the
+ * most recent run — *bits (device, NULL if no run used the filter), *words (uint32 words
+ * allocated, >= (n+31)/32), *anchor (the anchor vertex X, -1 if none).  A set bit v is a
+ * proof that v is in X's tree.  Synchronises the last run's stream. */
+ECL_CC_API ecl_cc_status ecl_cc_get_filter(ecl_cc_handle h, const uint32_t **bits,
+                                           int64_t *words, int32_t *anchor);
 
 /* Per-phase device time of the most recent full run with ECL_CC_OPT_TIMING set
  * (synchronises on it): ms[0] init_bin (incl. the counter memset), ms[1] hook_thread,

@@ -108,6 +108,9 @@ def _load(stats: bool = False) -> ctypes.CDLL:
             "ecl_cc_get_worklist": ([P, P, ctypes.POINTER(I64), P, ctypes.POINTER(I64)], INT),
             "ecl_cc_get_stats": ([P, ctypes.POINTER(I64)], INT),
             "ecl_cc_get_stats_ex": ([P, ctypes.POINTER(I64), INT], INT),
+            "ecl_cc_get_run_info": ([P, ctypes.POINTER(I64), INT], INT),
+            "ecl_cc_get_filter": ([P, ctypes.POINTER(P), ctypes.POINTER(I64),
+                                   ctypes.POINTER(I32)], INT),
             "ecl_cc_stats_enabled": ([], INT),
             "ecl_cc_get_timing": ([P, ctypes.POINTER(ctypes.c_float)], INT),
             "ecl_cc_status_string": ([INT], ctypes.c_char_p),
@@ -389,6 +392,20 @@ class Handle:
         self._check(self._lib.ecl_cc_get_worklist(self._h, _ptr(front), ctypes.byref(nf),
                                                   _ptr(back), ctypes.byref(nb)))
         return front, back
+
+    def run_info(self) -> dict:
+        """Decisions of the last run (ecl_cc_get_run_info)."""
+        arr = (ctypes.c_int64 * 4)()
+        self._check(self._lib.ecl_cc_get_run_info(self._h, arr, 4))
+        return {"lazy_init3": bool(arr[0]), "deep_forest_passes": bool(arr[1]),
+                "filter": bool(arr[2]), "anchor": int(arr[3])}
+
+    def filter_bitmap(self):
+        """(device address or None, words, anchor) of the R21 bitmap of the last run."""
+        b, w, a = ctypes.c_void_p(), ctypes.c_int64(0), ctypes.c_int32(-1)
+        self._check(self._lib.ecl_cc_get_filter(self._h, ctypes.byref(b), ctypes.byref(w),
+                                                ctypes.byref(a)))
+        return b.value, w.value, a.value
 
     def timing(self) -> dict:
         """Per-phase device milliseconds of the last run (needs set_option('timing', 1))."""

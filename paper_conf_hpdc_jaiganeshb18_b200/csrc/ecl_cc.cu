@@ -26,10 +26,6 @@ constexpr int kNumStats = 16;
 #define ECL_FAST_FINI 1
 #endif
 constexpr bool kFastFini = ECL_FAST_FINI != 0;   // Fini3 via finalize3_kernel
-#ifndef ECL_INIT_BRANGE
-#define ECL_INIT_BRANGE 1
-#endif
-constexpr bool kInitBlockRange = ECL_INIT_BRANGE != 0;   // init_bin: block-range mode
 
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
 
@@ -67,21 +63,12 @@ ecl_cc_status ensure_scratch(ecl_cc_handle h, int need, cudaStream_t s)
     if (h->wl) CK(cudaFreeAsync(h->wl, s), "cudaFreeAsync(wl)");
     if (h->ub) CK(cudaFreeAsync(h->ub, s), "cudaFreeAsync(ub)");
     if (h->tbits) CK(cudaFreeAsync(h->tbits, s), "cudaFreeAsync(tbits)");
-    if (h->scr) CK(cudaFreeAsync(h->scr, s), "cudaFreeAsync(scr)");
-    if (h->scru) CK(cudaFreeAsync(h->scru, s), "cudaFreeAsync(scru)");
     h->wl = nullptr;
     h->ub = nullptr;
     h->tbits = nullptr;
-    h->scr = nullptr;
-    h->scru = nullptr;
     h->cap = 0;
     CK(cudaMallocAsync((void **)&h->wl, sizeof(int) * (size_t)need, s), "cudaMallocAsync(wl)");
     CK(cudaMallocAsync((void **)&h->ub, sizeof(unsigned) * (size_t)need, s), "cudaMallocAsync(ub)");
-    if (kInitBlockRange) {
-        CK(cudaMallocAsync((void **)&h->scr, sizeof(int) * (size_t)need, s), "cudaMallocAsync(scr)");
-        CK(cudaMallocAsync((void **)&h->scru, sizeof(unsigned) * (size_t)need, s),
-           "cudaMallocAsync(scru)");
-    }
     CK(cudaMallocAsync((void **)&h->tbits, sizeof(unsigned) * (((size_t)need + 31) / 32), s),
        "cudaMallocAsync(tbits)");
     h->cap = need;
@@ -116,13 +103,15 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.t2 = h->t2;
     p.ttas = h->ttas;
     // R28: Init3 folded into the hook kernels (the separate pass over every row start is
-    // then a degree-only binning pass); auto = graphs with long rows (m >= 16 n), where
-    // that pass reads one sector per row for a few bytes
-    const int fuse = h->fuse_init == 2 ? (m >= 16LL * nrows ? 3 : 0) : h->fuse_init;
-    const bool lazy = h->init_mode == 3 && h->stop_after != 1 && fuse != 0;
-    p.lazy = !lazy ? 0 : fuse == 1 ? 1 : 2;
-    // every row lazy: the binning pass is Init1's (parent[v] = v, bins by degree)
-    p.init_mode = p.lazy == 1 ? 1 : h->init_mode;
+    // then a degree-only binning pass).  Auto: off for long rows (m >= 16 n: the R21
+    // filter needs Init3's forest), else decided on the device by the locality probe
+    // (random vertex IDs: on; meshes, whose Init3 chains R23 shortens: off)
+    const bool can = h->init_mode == 3 && h->stop_after != 1 && nrows > 0;
+    p.lazy = !can ? 0 : h->fuse_init == 1 ? 1
+           : (h->fuse_init == 2 && m < 16LL * nrows) ? 2 : 0;
+    p.lazy_flag = (const int *)(h->cnt + 7);
+    h->last_lazy = p.lazy;
+    p.init_mode = h->init_mode;
     p.jump = h->jump;
     p.batch = h->batch;
     p.anchor = h->cnt + 10;
@@ -133,6 +122,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     {
         // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
         const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
+        h->gbits_live = on;
         if (on) {
             const size_t words = ((size_t)n + 31) / 32;
             if (words > h->gbits_words) {
@@ -161,28 +151,19 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         auto k = identity_outside_kernel;
         k<<<grid_for(h, (const void *)k, n), kBlock, 0, s>>>(n, row_lo, row_lo + nrows, parent);
     }
+    if (p.lazy == 2)
+        locality_probe_kernel<idx_t><<<1, kBlock, 0, s>>>(row_lo, nrows, nindex, nlist,
+                                                           (int *)(h->cnt + 7));
     {
         auto k = init_bin_kernel<idx_t>;
-        const int grid = grid_for(h, (const void *)k,
-                                  ((long long)nrows + kInitPerThread - 1) / kInitPerThread);
-        p.scr = nullptr;
-        p.scru = nullptr;
-        p.rows_per_block = 0;
-        if (kInitBlockRange && h->scr) {
-            // each block owns a contiguous range of whole chunks (one worklist reservation
-            // per block instead of one per chunk)
-            const long long chunks = ((long long)nrows + kInitChunk - 1) / kInitChunk;
-            p.scr = h->scr;
-            p.scru = h->scru;
-            p.rows_per_block = (int)(((chunks + grid - 1) / grid) * kInitChunk);
-        }
-        k<<<grid, kBlock, 0, s>>>(p);
+        k<<<grid_for(h, (const void *)k, ((long long)nrows + kInitPerThread - 1) / kInitPerThread), kBlock, 0, s>>>(p);
     }
     if (h->prejump != 0 && h->stop_after != 1 && nrows > 0 && p.lazy != 1) {
         // R23: depth probe, then the passes (cooperative launch guarantees the
         // co-residency their grid barrier needs); both are no-ops on shallow forests
         int *ctl = (int *)(h->cnt + 4);
-        depth_probe_kernel<<<1, kBlock, 0, s>>>(row_lo, nrows, parent, ctl, h->prejump);
+        depth_probe_kernel<<<1, kBlock, 0, s>>>(row_lo, nrows, parent, ctl, h->prejump,
+                                                p.lazy ? p.lazy_flag : nullptr);
         auto k = prejump_kernel;
         const int blocks = std::min(h->sms * blocks_per_sm(h, (const void *)k, 0),
                                     (int)std::max(1LL, ((long long)nrows + kBlock - 1) / kBlock));
@@ -383,7 +364,7 @@ ecl_cc_status ecl_cc_destroy(ecl_cc_handle h)
         cudaStream_t s = h->side;
         if (h->done_valid) cudaStreamWaitEvent(s, h->done, 0);
         void *bufs[] = {h->wl, h->ub, h->tbits, h->cnt, h->flags, h->e2e_index, h->e2e_list,
-                        h->e2e_labels, h->gbits, h->csr_tmp, h->scr, h->scru};
+                        h->e2e_labels, h->gbits, h->csr_tmp};
         for (void *b : bufs)
             if (b) cudaFreeAsync(b, s);
         cudaStreamSynchronize(s);
@@ -616,7 +597,7 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
         // ranks can hold long chains of former roots, which Fini3 would walk per vertex)
         int *ctl = (int *)(h->cnt + 4);
         CK(cudaMemsetAsync(ctl, 0, 4 * sizeof(unsigned long long), s), "memset ctl");
-        depth_probe_kernel<<<1, kBlock, 0, s>>>(0, n, parent, ctl, h->flatten_passes);
+        depth_probe_kernel<<<1, kBlock, 0, s>>>(0, n, parent, ctl, h->flatten_passes, nullptr);
         auto k = prejump_kernel;
         const int blocks = std::min(h->sms * blocks_per_sm(h, (const void *)k, 0),
                                     (int)std::max(1LL, ((long long)n + kBlock - 1) / kBlock));
@@ -804,7 +785,7 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         h->prejump = (int)value;
         break;
     case ECL_CC_OPT_FUSE_INIT:
-        if (value < 0 || value > 3) return fail_arg(h, "fuse_init must be 0..3");
+        if (value < 0 || value > 2) return fail_arg(h, "fuse_init must be 0, 1 or 2");
         h->fuse_init = (int)value;
         break;
     case ECL_CC_OPT_FLATTEN_PASSES:
@@ -849,6 +830,38 @@ ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, int64_t *nfro
         CK(cudaMemcpyAsync(back, h->wl + h->cap - nb, sizeof(int) * nb, cudaMemcpyDeviceToDevice, s),
            "D2D back");
     CK(cudaStreamSynchronize(s), "sync");
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_get_run_info(ecl_cc_handle h, int64_t *out, int count)
+{
+    if (!h || !out || count < 0 || count > 4) return ECL_CC_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
+    unsigned long long c[11] = {};
+    CK(cudaStreamSynchronize(h->last_stream), "sync");
+    CK(cudaMemcpy(c, h->cnt, sizeof(c), cudaMemcpyDeviceToHost), "D2H counters");
+    const int *ctl = (const int *)(c + 4);
+    const int lazy_flag = (int)(unsigned)c[7];
+    const int64_t v[4] = {h->last_lazy == 1 || (h->last_lazy == 2 && lazy_flag) ? 1 : 0,
+                          ctl[0] ? 1 : 0, h->gbits_live ? 1 : 0,
+                          c[10] ? (int64_t)(unsigned)c[10] : -1};
+    for (int i = 0; i < count; i++) out[i] = v[i];
+    return ECL_CC_OK;
+}
+
+ecl_cc_status ecl_cc_get_filter(ecl_cc_handle h, const uint32_t **bits, int64_t *words,
+                                int32_t *anchor)
+{
+    if (!h || !bits || !words || !anchor) return ECL_CC_ERR_INVALID_ARG;
+    DeviceGuard g(h->device);
+    *bits = h->gbits_live ? h->gbits : nullptr;
+    *words = h->gbits_live ? (int64_t)h->gbits_words : 0;
+    *anchor = -1;
+    if (!h->gbits_live) return ECL_CC_OK;
+    unsigned long long a = 0;
+    CK(cudaStreamSynchronize(h->last_stream), "sync");
+    CK(cudaMemcpy(&a, h->cnt + 10, sizeof(a), cudaMemcpyDeviceToHost), "D2H anchor");
+    *anchor = a ? (int32_t)(unsigned)a : -1;
     return ECL_CC_OK;
 }
 

@@ -16,8 +16,6 @@ struct ecl_cc_ctx {
     int *wl = nullptr;
     unsigned *ub = nullptr;
     unsigned *tbits = nullptr;            // R24 thread-bin work bitmap (one bit per row)
-    int *scr = nullptr;                   // init_bin's per-block worklist staging (vertex,
-    unsigned *scru = nullptr;             //   block-local unit base), cap entries each
     int cap = 0;
     unsigned long long *cnt = nullptr;    // [0..1] worklist counters, [8..9] int
                                           // scheduling counters, [10] R21 anchor,
@@ -54,6 +52,8 @@ struct ecl_cc_ctx {
     size_t csr_tmp_bytes = 0;
     unsigned *gbits = nullptr;            // R21 bitmap (grow-only)
     size_t gbits_words = 0;
+    bool gbits_live = false;              // the last run used the R21 bitmap
+    int last_lazy = 0;                    // the last run's R28 mode (0 off, 1 on, 2 probe)
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks

@@ -64,6 +64,30 @@ def depth_stats(parent):
             "nonroots": int(nonroot.sum())}
 
 
+def filter_coverage(h, forest, n):
+    """After a local run: the share of the anchor's class (vertices whose root equals the
+    anchor's) already marked in the handle's R21 bitmap — the walks a bitmap-assisted
+    flatten would skip."""
+    from cuda.bindings import runtime as cudart
+    ptr, words, anchor = h.filter_bitmap()
+    if not ptr or anchor < 0:
+        return None
+    nw = (n + 31) // 32
+    bits = torch.empty(nw, dtype=torch.int32, device="cuda")
+    cudart.cudaMemcpy(bits.data_ptr(), ptr, nw * 4, cudart.cudaMemcpyKind.cudaMemcpyDeviceToDevice)
+    f = forest.clone()
+    h.finalize(f)
+    ar = torch.arange(n, device="cuda")
+    b = ((bits.to(torch.int64)[ar // 32] >> (ar % 32)) & 1).bool()
+    cls = f == f[anchor]
+    nonroot = f != ar
+    return {"anchor_class": int(cls.sum()), "marked": int((b & cls).sum()),
+            "marked_outside_class": int((b & ~cls).sum()),
+            "coverage": round(float((b & cls).sum()) / max(int(cls.sum()), 1), 4),
+            "nonroots": int(nonroot.sum()),
+            "nonroots_outside_class": int((nonroot & ~cls).sum())}
+
+
 def tree_merge(h, forests, G, n, args, ref, t_rank):
     rounds = {}
     for (rd, send, recv) in edist.tree_schedule(G):
@@ -203,7 +227,7 @@ def main():
     res["partition"] = "entries" if args.even else "row_weights"
     for G in [int(x) for x in args.gpus.split(",")]:
         bounds = edist.partition_rows(nidx64.cpu(), G, weights=wts)
-        forests, t_rank = [], []
+        forests, t_rank, cov = [], [], []
         for r in range(G):
             lo, hi = bounds[r], bounds[r + 1]
             idx, lst = edist.slice_rows(nidx64, g.nlist, lo, hi)
@@ -211,6 +235,8 @@ def main():
             t, _ = timed(lambda: h.run_rows(n, lo, hi, idx, lst, parent=par, flatten=(G == 1)))
             t_rank.append(t)
             forests.append(par)
+            if G > 1:
+                cov.append(filter_coverage(h, par, n))
             del idx, lst
         if args.calibrate and G > 1 and wts is not None:
             # one measured step re-weights the rows (dist.rebalance_weights), then the
@@ -233,7 +259,8 @@ def main():
                    [round(x, 4) for x in t_first] if args.calibrate and G > 1 else None,
                "rank_entries": [int(nidx64[bounds[r + 1]] - nidx64[bounds[r]]) for r in range(G)],
                "rank_rows": [bounds[r + 1] - bounds[r] for r in range(G)],
-               "rank_depth": [depth_stats(f) for f in forests] if G > 1 else None}
+               "rank_depth": [depth_stats(f) for f in forests] if G > 1 else None,
+               "rank_filter_coverage": cov or None}
         if "tree" in args.merge and G > 1:
             tf = [f.clone() for f in forests]
             row["tree"] = tree_merge(h, tf, G, n, args, ref, t_rank)
