@@ -356,15 +356,13 @@ def launches_per_step(world: int, rank: int, chunks: int, merge: str, probe: int
     shallow forests), hook_thread, hook_range x2, finalize (+ `probe`: R28's locality
     probe, launched when m < 16n); with G ranks: identity_outside
     instead of finalize in run_rows, then for the tree merge one merge_hook per received
-    chunk and rank 0's finalize; for the encoded merges a flatten (R23 depth probe +
-    passes + finalize) and encode on every rank g > 0, and on rank 0 a flatten,
-    merge_bits + merge_pairs, and a flatten."""
+    chunk and rank 0's finalize; for the encoded merges encode on every rank g > 0, and
+    merge_bits + merge_pairs + finalize on rank 0."""
     if world == 1:
         return 7 + probe
     from paper_conf_hpdc_jaiganeshb18_b200 import dist as edist
     if merge != "tree":
-        fl = 3 if edist.EncodedMerge.FLATTEN.get("flatten_passes") else 1
-        return 7 + (2 * fl + 2 if rank == 0 else fl + 1)
+        return 7 + (3 if rank == 0 else 1)
     recv = sum(1 for (_, _s, r) in edist.tree_schedule(world) if r == rank)
     return 7 + recv * chunks + (1 if rank == 0 else 0)
 
@@ -380,7 +378,7 @@ def main():
     ap.add_argument("--load-mode", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--chunks", type=int, default=4, help="tree merge: chunks per round")
-    ap.add_argument("--calibrate", type=int, default=1,
+    ap.add_argument("--calibrate", type=int, default=0,
                     help="N > 1: re-partition once from measured local-forest times")
     ap.add_argument("--merge", default="p2p", choices=["p2p", "compact", "tree"],
                     help="N > 1: forest merge (dist.EncodedMerge p2p / compact, or the "

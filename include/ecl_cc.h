@@ -184,13 +184,16 @@ ECL_CC_API ecl_cc_status ecl_cc_merge(ecl_cc_handle h, int32_t n, int32_t v_lo, 
 ECL_CC_API ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void *stream);
 
 /* ---- encoded forest exchange and P2P merge (not in the paper) ----------
- * ecl_cc_forest_encode: encode a FLATTENED labelling `labels` (n entries, labels[v] the
- *   root of v's tree, e.g. the output of ecl_cc_run_rows without STOP_AFTER 2, or of
- *   ecl_cc_finalize) as the relation it spans: D = labels[anchor] (pick a vertex of the
- *   largest component, e.g. the highest-degree row; anchor = -1: no bitmap class, every
- *   non-root becomes a pair), bits[v / 32] bit v % 32 set iff
- *   labels[v] == D, and the pairs (v, labels[v]) of every other v with labels[v] != v.
- *   The edges {(v, D) : bit v} u {(v, labels[v]) : pairs} span exactly the classes of
+ * ecl_cc_forest_encode: encode a forest `labels` (n entries with labels[x] <= x in x's
+ *   tree: a flattened labelling, or an unflattened forest such as ecl_cc_run_rows with
+ *   STOP_AFTER 2 leaves — each vertex's root is then found by a read-only walk) as the
+ *   relation it spans: D = root(anchor) (pick a vertex of the largest component, e.g. the
+ *   highest-degree row; anchor = -1: no bitmap class, every non-root becomes a pair;
+ *   with ECL_CC_OPT_MERGE_FILTER set and an R21 bitmap in this handle's most recent run,
+ *   which must be the run that built `labels`, that run's anchor replaces `anchor` and its
+ *   bitmap proves most vertices' class without a walk), bits[v / 32] bit v % 32 set iff
+ *   root(v) == D, and the pairs (v, root(v)) of every other v with root(v) != v.
+ *   The edges {(v, D) : bit v} u {(v, root(v)) : pairs} span exactly the classes of
  *   `labels`, so merging them is exact (hook-once sufficiency).
  *     bits   (n + 31) / 32 uint32 words out (device)
  *     pairs  2 x cap int32 out (device): pair i is (pairs[2i], pairs[2i+1]); the order is
@@ -282,7 +285,7 @@ typedef enum {
                                      1 always, 2 when a depth probe finds the forest deep.
                                      For merged multi-GPU forests, whose former roots
                                      form long chains that Fini3 would walk per vertex. */
-    ECL_CC_OPT_FUSE_INIT = 19     /* Init3 folded into the hook kernels (R28):
+    ECL_CC_OPT_FUSE_INIT = 19,    /* Init3 folded into the hook kernels (R28):
                                      the init kernel only bins rows by degree and writes
                                      parent[v] = v; the kernel that owns a row's start
                                      CASes parent[v] from v to the first smaller
@@ -299,6 +302,14 @@ typedef enum {
                                      the R23 passes are skipped.  Labels unchanged (R13);
                                      the worklists then hold every row of their degree
                                      range, not only rows with a smaller neighbour.    */
+    ECL_CC_OPT_MERGE_FILTER = 20  /* multi-GPU: 1 = ecl_cc_forest_encode,
+                                     ecl_cc_merge_encoded and
+                                     ecl_cc_finalize treat `parent` as the forest this
+                                     handle's most recent run built and use that run's
+                                     R21 bitmap (anchor-tree membership proofs) to skip
+                                     walks; merge_encoded extends the bitmap with the
+                                     vertices it joins to the anchor's tree.  0 (default)
+                                     = no such assumption.                             */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

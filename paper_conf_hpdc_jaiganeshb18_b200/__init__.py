@@ -47,6 +47,7 @@ OPT = {
     "prejump": 17,
     "flatten_passes": 18,
     "fuse_init": 19,
+    "merge_filter": 20,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

@@ -469,8 +469,13 @@ ecl_cc_status ecl_cc_forest_encode(ecl_cc_handle h, int32_t n, const int32_t *la
     CK(cudaMemsetAsync(meta, 0, sizeof(uint64_t), s), "memset meta");
     auto k = encode_kernel;
     const long long words = ((long long)n + kWarp - 1) / kWarp;
+    // ECL_CC_OPT_MERGE_FILTER: `labels` is the forest this handle's last run built; that
+    // run's R21 bitmap and anchor (which then replaces `anchor`) prove most vertices'
+    // class without a walk
+    const bool filt = h->merge_filter && h->gbits_live;
     k<<<grid_for(h, (const void *)k, words * kWarp), kBlock, 0, s>>>(
-        n, labels, anchor, bits, pairs, cap, (unsigned long long *)meta);
+        n, labels, anchor, bits, pairs, cap, (unsigned long long *)meta,
+        filt ? h->gbits : nullptr, h->cnt + 10);
     CK(cudaGetLastError(), "encode launch");
     return end_call(h, s);
 }
@@ -506,14 +511,17 @@ ecl_cc_status ecl_cc_merge_encoded(ecl_cc_handle h, int32_t n, int npeers,
 #else
 #define ECL_SA
 #endif
+    unsigned *filt = (h->merge_filter && h->gbits_live) ? h->gbits : nullptr;
     if (h->load_mode == 1) {
         auto kb = merge_bits_kernel<1>;
-        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas ECL_SA);
+        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas,
+                                                                            filt, h->cnt + 10 ECL_SA);
         auto kp = merge_pairs_kernel<1>;
         kp<<<grid_for(h, (const void *)kp, -1), kBlock, 0, s>>>(ps, parent, h->ttas ECL_SA);
     } else {
         auto kb = merge_bits_kernel<0>;
-        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas ECL_SA);
+        kb<<<grid_for(h, (const void *)kb, words * kWarp), kBlock, 0, s>>>(n, ps, parent, h->ttas,
+                                                                            filt, h->cnt + 10 ECL_SA);
         auto kp = merge_pairs_kernel<0>;
         kp<<<grid_for(h, (const void *)kp, -1), kBlock, 0, s>>>(ps, parent, h->ttas ECL_SA);
     }
@@ -607,7 +615,13 @@ ecl_cc_status ecl_cc_finalize(ecl_cc_handle h, int32_t n, int32_t *parent, void 
         CK(cudaLaunchCooperativeKernel((const void *)k, dim3(blocks), dim3(kBlock), args, 0, s),
            "flatten passes launch");
     }
-    if (h->fini == 3 && kFastFini) {
+    if (h->merge_filter && h->gbits_live && h->fini == 3) {
+        // the R21 bitmap of the run that built `parent` (extended by merge_bits) proves
+        // most vertices' root without a walk
+        auto k = finalize_filter_kernel;
+        k<<<grid_for(h, (const void *)k, ((long long)n + kWarp - 1) / kWarp * kWarp), kBlock, 0, s>>>(
+            n, parent, h->gbits, h->cnt + 10);
+    } else if (h->fini == 3 && kFastFini) {
         auto k = finalize3_kernel<0>;
         k<<<grid_for(h, (const void *)k, ((long long)n + kFinPer - 1) / kFinPer), kBlock, 0, s>>>(n, parent);
     } else {
@@ -783,6 +797,9 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_PREJUMP:
         if (value < 0 || value > 2) return fail_arg(h, "prejump must be 0, 1 or 2");
         h->prejump = (int)value;
+        break;
+    case ECL_CC_OPT_MERGE_FILTER:
+        h->merge_filter = value != 0;
         break;
     case ECL_CC_OPT_FUSE_INIT:
         if (value < 0 || value > 2) return fail_arg(h, "fuse_init must be 0, 1 or 2");

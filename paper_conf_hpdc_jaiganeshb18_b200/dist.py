@@ -174,11 +174,14 @@ class EncodedMerge:
     """Flat merge of encoded forests into rank 0 (the variants the survey
     lists beside the binomial tree of full forests).
 
-    Every rank g != 0 flattens its local forest (ecl_cc_finalize), encodes it
-    (ecl_cc_forest_encode: an n/32-word bitmap of "label == D" plus the pairs (v, L[v]) of
-    the remaining non-roots — for a power-law graph 16 MB + a few MB instead of the 537 MB
-    label array at n = 2^27), and rank 0 hooks all peers' relations in one
-    ecl_cc_merge_encoded call, then flattens once.  Exact by hook-once sufficiency
+    Every rank g != 0 encodes its (unflattened) local forest (ecl_cc_forest_encode: an
+    n/32-word bitmap of "root == D" plus the pairs (v, root(v)) of the remaining non-roots
+    — for a power-law graph 16 MB + a few MB instead of the 537 MB parent array at
+    n = 2^27), and rank 0 hooks all peers' relations into its own local forest in one
+    ecl_cc_merge_encoded call, then flattens once.  With ECL_CC_OPT_MERGE_FILTER every
+    step uses the R21 anchor bitmap of the rank's own local run as membership proofs, so
+    most vertices of the giant tree need no random walk (the walks of a local forest's
+    flatten are random DRAM reads at n = 2^27).  Exact by hook-once sufficiency
     (P:L161-L163): the encoded edges span the same classes as the labels.
 
     mode "compact": the encodings travel over the process group (NCCL send/recv; gloo
@@ -193,18 +196,15 @@ class EncodedMerge:
       gloo (tests, one GPU) the streams are synchronised around host messages.
     """
 
-    # ecl_cc_finalize options of the flattens: a local forest's vertices outside the rank's
-    # rows hang below chains of former roots (each hooked once, never walked again), so a
-    # plain Fini3 walk per vertex is slow; the R23 pointer-jumping passes first shorten
-    # every chain (ECL_CC_OPT_FLATTEN_PASSES)
-    FLATTEN = {"fini": 3, "flatten_passes": 1}
+    # handle options around the merge's calls (restored afterwards)
+    OPTS = {"merge_filter": 1}
 
     def __init__(self, handle, n: int, anchor: int, mode: str = "p2p", group=None,
-                 flatten: Optional[dict] = None):
+                 opts: Optional[dict] = None):
         if mode not in ("compact", "p2p"):
             raise ValueError(mode)
         self.h, self.n, self.anchor, self.mode, self.group = handle, n, anchor, mode, group
-        self.flatten = dict(self.FLATTEN if flatten is None else flatten)
+        self.opts = dict(self.OPTS if opts is None else opts)
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
         if self.world - 1 > 8:
@@ -229,13 +229,14 @@ class EncodedMerge:
         elif self.rank == 0:
             self.recv = [handle.encode_buffers(n) for _ in range(1, self.world)]
 
-    def _flatten(self, parent):
-        for k, v in self.flatten.items():
+    def _with_opts(self, fn, *a):
+        for k, v in self.opts.items():
             self.h.set_option(k, v)
         try:
-            self.h.finalize(parent)
+            return fn(*a)
         finally:
-            self.h.set_option("fini", 3).set_option("flatten_passes", 0)
+            for k in self.opts:
+                self.h.set_option(k, 0)
 
     def close(self):
         for p in self.mapped:
@@ -259,10 +260,9 @@ class EncodedMerge:
     def __call__(self, parent: torch.Tensor, broadcast: bool = False):
         h, rank = self.h, self.rank
         if self.world == 1:
-            self._flatten(parent)
+            self._with_opts(h.finalize, parent)
         elif rank != 0:
-            self._flatten(parent)                           # labels = roots
-            h.forest_encode(parent, self.anchor, self.enc)
+            self._with_opts(h.forest_encode, parent, self.anchor, self.enc)
             if self.mode == "p2p":
                 self._send(self.flag, 0)                    # "my encoding is complete"
                 self._recv(self.flag, 0)                    # rank 0 finished reading it
@@ -274,11 +274,10 @@ class EncodedMerge:
                 if npairs:
                     self._send(self.enc["pairs"][:2 * npairs], 0)
         else:
-            self._flatten(parent)              # the merge's finds are then one hop long
             if self.mode == "p2p":
                 for r in range(1, self.world):
                     self._recv(self.flag, r)
-                h.merge_encoded(parent, self.peers)
+                self._with_opts(h.merge_encoded, parent, self.peers)
                 if self.gloo:
                     torch.cuda.current_stream(parent.device).synchronize()
                 for r in range(1, self.world):
@@ -293,8 +292,8 @@ class EncodedMerge:
                         self._recv(buf["pairs"][:2 * npairs], r)
                     peers.append({"bits": buf["bits"], "pairs": buf["pairs"],
                                   "meta": buf["meta"], "cap": npairs})
-                h.merge_encoded(parent, peers)
-            self._flatten(parent)
+                self._with_opts(h.merge_encoded, parent, peers)
+            self._with_opts(h.finalize, parent)
         if broadcast:
             if self.gloo and parent.is_cuda:
                 host = parent.cpu()

@@ -36,7 +36,8 @@ def _make(name, sd, seed, loopdup):
     return gg.inject_loops_dups(g, seed=seed) if loopdup else g
 
 
-def _worker(rank, world, port, name, sd, seed, chunks, broadcast, loopdup, variant, q):
+def _worker(rank, world, port, name, sd, seed, chunks, broadcast, loopdup, variant, q,
+            filt=2):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -53,6 +54,7 @@ def _worker(rank, world, port, name, sd, seed, chunks, broadcast, loopdup, varia
         n = g.n
         del g
         with ecl.Handle(0) as h:
+            h.set_option("filter", filt)
             parent = h.run_rows(n, lo, hi, idx, lst, flatten=False)
             if variant == "tree":
                 out = edist.forest_merge(parent, h, chunks=chunks, broadcast=broadcast)
@@ -73,12 +75,12 @@ def _worker(rank, world, port, name, sd, seed, chunks, broadcast, loopdup, varia
 
 
 def run_world(world, name, sd, seed, chunks=2, broadcast=False, loopdup=False,
-              variant="tree"):
+              variant="tree", filt=2):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
     procs = [ctx.Process(target=_worker, args=(r, world, port, name, sd, seed, chunks,
-                                               broadcast, loopdup, variant, q))
+                                               broadcast, loopdup, variant, q, filt))
              for r in range(world)]
     for p in procs:
         p.start()
@@ -126,3 +128,11 @@ def test_multiprocess_encoded_merge(variant, world, name, sd):
 @pytest.mark.parametrize("variant", ["compact", "p2p"])
 def test_multiprocess_encoded_merge_broadcast_raw(variant):
     run_world(3, "C4", 8, seed=21, broadcast=True, loopdup=True, variant=variant)
+
+
+@pytest.mark.parametrize("variant", ["compact", "p2p"])
+@pytest.mark.parametrize("world", [2, 4])
+def test_multiprocess_encoded_merge_with_filter(variant, world):
+    """The R21 bitmap of each rank's own local run as membership proofs in the encode, the
+    merge and the final flatten (forced on: auto only enables it for 4n > 128 MB)."""
+    run_world(world, "C5", 9, seed=world + 30, variant=variant, filt=1)

@@ -651,5 +651,37 @@ def test_fuse_init_auto_decision(h):
         assert_parity(h, g)
         info = h.run_info()
         assert info["lazy_init3"] == lazy, (name, info)
-        if name == "C2":
-            assert info["deep_forest_passes"]
+
+
+@pytest.mark.parametrize("G", [2, 4, 9])
+@pytest.mark.parametrize("name", ["C4", "C5"])
+@pytest.mark.parametrize("filt", [0, 1])
+def test_fake_multi_gpu_encoded_merge_filter(name, G, filt):
+    """dist.EncodedMerge's flow with one handle per fake rank: unflattened local forests
+    (R21 filter forced on), peers encode with their own run's bitmap as membership proofs
+    (ECL_CC_OPT_MERGE_FILTER), rank 0 merges into its own unflattened forest and flattens
+    with its bitmap (extended by the merge)."""
+    from paper_conf_hpdc_jaiganeshb18_b200 import dist
+    g = gg.make_config(name, seed=17, scale_down=SMALL[name] + 1, device="cuda")
+    expect, _ = oracle.bfs(*g.numpy())
+    nindex64 = g.nindex.to(torch.int64)
+    bounds = dist.partition_rows(nindex64, G, weights=dist.row_weights(nindex64, g.nlist))
+    hs = [ecl.Handle(0) for _ in range(G)]
+    try:
+        forests, encs = [], []
+        for r in range(G):
+            hs[r].set_option("filter", 1).set_option("merge_filter", filt)
+            idx, lst = dist.slice_rows(nindex64, g.nlist, bounds[r], bounds[r + 1])
+            f = hs[r].run_rows(g.n, bounds[r], bounds[r + 1], idx, lst, flatten=False)
+            forests.append(f)
+            if r > 0:
+                enc = hs[r].encode_buffers(g.n)
+                hs[r].forest_encode(f, dist.row_anchor(idx, bounds[r]), enc)
+                encs.append(enc)
+        hs[0].merge_encoded(forests[0], encs)
+        hs[0].finalize(forests[0])
+        torch.cuda.synchronize()
+        assert np.array_equal(forests[0].cpu().numpy(), expect)
+    finally:
+        for x in hs:
+            x.close()

@@ -109,14 +109,10 @@ def tree_merge(h, forests, G, n, args, ref, t_rank):
                                           "round_ms": round(rt, 4)})
         del base
     fins = {}
-    for name in ("fini3", "passes"):
-        set_flatten(h, name)
-        f = forests[0].clone()
-        fins[name], _ = timed(lambda: h.finalize(f), reps=1)
-        del f
-    set_flatten(h, "passes")
+    f = forests[0].clone()
+    fins["fini3"], _ = timed(lambda: h.finalize(f), reps=1)
+    del f
     h.finalize(forests[0])
-    set_flatten(h, "fini3")
     t_fin = min(fins.values())
     torch.cuda.synchronize()
     ok = bool(torch.equal(forests[0], ref))
@@ -127,76 +123,80 @@ def tree_merge(h, forests, G, n, args, ref, t_rank):
             "projected_ms": round(max(t_rank) + t_rounds + t_fin, 4)}
 
 
-FLATTEN = {"fini3": dict(fini=3, flatten_passes=0), "fini1": dict(fini=1, flatten_passes=0),
-           "fini2": dict(fini=2, flatten_passes=0), "passes": dict(fini=3, flatten_passes=1)}
+def snapshot_filter(h, n):
+    """Copy of a handle's R21 bitmap (merge_bits extends it: restore between timings)."""
+    from cuda.bindings import runtime as cudart
+    ptr, words, anchor = h.filter_bitmap()
+    if not ptr:
+        return None
+    nw = (n + 31) // 32
+    buf = torch.empty(nw, dtype=torch.int32, device="cuda")
+    cudart.cudaMemcpy(buf.data_ptr(), ptr, nw * 4, cudart.cudaMemcpyKind.cudaMemcpyDeviceToDevice)
+    return ptr, buf
 
 
-def set_flatten(h, name):
-    for k, v in FLATTEN[name].items():
-        h.set_option(k, v)
+def restore_filter(snap):
+    from cuda.bindings import runtime as cudart
+    if snap is not None:
+        ptr, buf = snap
+        cudart.cudaMemcpy(ptr, buf.data_ptr(), buf.numel() * 4,
+                          cudart.cudaMemcpyKind.cudaMemcpyDeviceToDevice)
 
 
-def encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank):
-    """Every rank flattens its local forest (variants of ecl_cc_finalize timed: Fini3,
-    Fini1, Fini2, R23 passes + Fini3), ranks g > 0 encode; rank 0 merges all encodings in
-    one ecl_cc_merge_encoded call on its flattened forest and flattens once more."""
-    flat_ms = {}
-    for name in FLATTEN:
-        set_flatten(h, name)
-        per = []
-        for r in range(G):
-            f = forests[r].clone()
-            t_copy, _ = timed(lambda: f.copy_(forests[r]))
-            t, _ = timed(lambda: (f.copy_(forests[r]), h.finalize(f)))
-            per.append(round(max(t - t_copy, 0.0), 4))
-            del f
-        flat_ms[name] = per
-    best = min(flat_ms, key=lambda k: max(flat_ms[k]))
-    set_flatten(h, best)
-    flat = []
-    for r in range(G):
-        f = forests[r].clone()
-        h.finalize(f)
-        flat.append(f)
+def encoded_merge(hs, forests, G, n, bounds, nidx64, args, ref, t_rank, use_filter):
+    """dist.EncodedMerge on one GPU: ranks g > 0 encode their unflattened local forest
+    (ECL_CC_OPT_MERGE_FILTER: with their own run's R21 bitmap as membership proofs), rank 0
+    merges all encodings into its own local forest and flattens."""
+    for h in hs:
+        h.set_option("merge_filter", 1 if use_filter else 0)
     encs, t_enc, pair_counts = [], [], []
     for r in range(1, G):
         idx = nidx64[bounds[r]:bounds[r + 1] + 1]
         anchor = edist.row_anchor(idx, bounds[r])
-        enc = h.encode_buffers(n)
-        t, _ = timed(lambda: h.forest_encode(flat[r], anchor, enc))
+        enc = hs[r].encode_buffers(n)
+        t, _ = timed(lambda: hs[r].forest_encode(forests[r], anchor, enc))
         t_enc.append(t)
         pair_counts.append(int(enc["meta"][0]))
         encs.append(enc)
-    base = flat[0].clone()
+    h0 = hs[0]
+    base = forests[0].clone()
+    snap = snapshot_filter(h0, n) if use_filter else None
+    f = forests[0]
 
     def mrg():
-        flat[0].copy_(base)
-        h.merge_encoded(flat[0], encs)
-    copy_t, _ = timed(lambda: flat[0].copy_(base))
-    t_m, _ = timed(mrg)
-    t_m = max(t_m - copy_t, 0.0)
-    hs = ecl.Handle(0, stats=True)
-    f = base.clone()
-    hs.merge_encoded(f, encs)
-    merge_stats = hs.stats()
-    del f, hs
-    flat[0].copy_(base)
-    h.merge_encoded(flat[0], encs)
-    set_flatten(h, "fini3")
-    t_fin, _ = timed(lambda: h.finalize(flat[0]), reps=1)
+        f.copy_(base)
+        restore_filter(snap)
+        h0.merge_encoded(f, encs)
+        h0.finalize(f)
+    copy_t, _ = timed(lambda: (f.copy_(base), restore_filter(snap)))
+    t_all, _ = timed(mrg)
+    f.copy_(base)
+    restore_filter(snap)
+    h0.merge_encoded(f, encs)
     torch.cuda.synchronize()
-    ok = bool(torch.equal(flat[0], ref))
+    a, b = torch.cuda.Event(True), torch.cuda.Event(True)
+    a.record()
+    h0.finalize(f)
+    b.record()
+    b.synchronize()
+    t_fin = a.elapsed_time(b)
+    t_m = max(t_all - copy_t - t_fin, 0.0)
+    ok = bool(torch.equal(f, ref))
+    f.copy_(base)
+    restore_filter(snap)
+    for h in hs:
+        h.set_option("merge_filter", 0)
     enc_bytes = sum(((n + 31) // 32) * 4 + 16 + 8 * c for c in pair_counts)
     xfer = enc_bytes / (args.link_gbs * 1e9) * 1e3
-    ready = max([t_rank[0] + flat_ms[best][0]] +
-                [t_rank[r] + flat_ms[best][r] + t_enc[r - 1] for r in range(1, G)])
+    ready = max([t_rank[0]] + [t_rank[r] + t_enc[r - 1] for r in range(1, G)])
     p2p = ready + max(t_m, xfer) + t_fin
     compact = ready + xfer + t_m + t_fin
-    return {"flatten_ms": flat_ms, "flatten_used": best, "merge_stats": merge_stats,
-            "encode_ms": [round(x, 4) for x in t_enc], "pairs": pair_counts,
-            "encoded_bytes_total": enc_bytes, "merge_ms": round(t_m, 4),
-            "transfer_ms_model": round(xfer, 4), "final_flatten_ms": round(t_fin, 4),
-            "merge_total_p2p_ms": round(max(t_m, xfer) + t_fin, 4),
+    return {"filter": use_filter, "encode_ms": [round(x, 4) for x in t_enc],
+            "pairs": pair_counts, "encoded_bytes_total": enc_bytes,
+            "merge_ms": round(t_m, 4), "transfer_ms_model": round(xfer, 4),
+            "final_flatten_ms": round(t_fin, 4),
+            "merge_plus_flatten_ms": round(max(t_m, xfer) + t_fin, 4),
+            "encode_merge_flatten_ms": round(max(t_enc or [0]) + max(t_m, xfer) + t_fin, 4),
             "projected_ms": round(p2p, 4), "projected_compact_ms": round(compact, 4),
             "labels_exact": ok}
 
@@ -210,7 +210,7 @@ def main():
     ap.add_argument("--even", action="store_true")
     ap.add_argument("--order", type=int, default=2, help="ECL_CC_OPT_ORDER of every run")
     ap.add_argument("--merge", default="tree,encoded")
-    ap.add_argument("--calibrate", type=int, default=1,
+    ap.add_argument("--calibrate", type=int, default=0,
                     help="re-partition once from the measured local-forest times")
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=1, device="cuda")
@@ -228,15 +228,19 @@ def main():
     for G in [int(x) for x in args.gpus.split(",")]:
         bounds = edist.partition_rows(nidx64.cpu(), G, weights=wts)
         forests, t_rank, cov = [], [], []
+        hs = [h] + [ecl.Handle(0) for _ in range(G - 1)]     # one handle per rank
+        for hh in hs:
+            hh.set_option("order", args.order)
         for r in range(G):
             lo, hi = bounds[r], bounds[r + 1]
             idx, lst = edist.slice_rows(nidx64, g.nlist, lo, hi)
             par = torch.empty(n, dtype=torch.int32, device="cuda")
-            t, _ = timed(lambda: h.run_rows(n, lo, hi, idx, lst, parent=par, flatten=(G == 1)))
+            t, _ = timed(lambda: hs[r].run_rows(n, lo, hi, idx, lst, parent=par,
+                                                flatten=(G == 1)))
             t_rank.append(t)
             forests.append(par)
             if G > 1:
-                cov.append(filter_coverage(h, par, n))
+                cov.append(filter_coverage(hs[r], par, n))
             del idx, lst
         if args.calibrate and G > 1 and wts is not None:
             # one measured step re-weights the rows (dist.rebalance_weights), then the
@@ -250,7 +254,8 @@ def main():
                 lo, hi = bounds[r], bounds[r + 1]
                 idx, lst = edist.slice_rows(nidx64, g.nlist, lo, hi)
                 par = torch.empty(n, dtype=torch.int32, device="cuda")
-                t, _ = timed(lambda: h.run_rows(n, lo, hi, idx, lst, parent=par, flatten=False))
+                t, _ = timed(lambda: hs[r].run_rows(n, lo, hi, idx, lst, parent=par,
+                                                    flatten=False))
                 t_rank.append(t)
                 forests.append(par)
                 del idx, lst
@@ -266,14 +271,20 @@ def main():
             row["tree"] = tree_merge(h, tf, G, n, args, ref, t_rank)
             del tf
         if "encoded" in args.merge and G > 1:
-            row["encoded"] = encoded_merge(h, forests, G, n, bounds, nidx64, args, ref, t_rank)
+            row["encoded"] = encoded_merge(hs, forests, G, n, bounds, nidx64, args, ref,
+                                           t_rank, False)
+            row["encoded_filter"] = encoded_merge(hs, forests, G, n, bounds, nidx64, args,
+                                                  ref, t_rank, True)
         if G == 1:
             row["projected_ms"] = round(t_rank[0], 4)
-        best = min([row[k]["projected_ms"] for k in ("tree", "encoded") if k in row] or
+        best = min([row[k]["projected_ms"] for k in ("tree", "encoded", "encoded_filter")
+                    if k in row] or
                    [row.get("projected_ms", t_rank[0])])
         row["projected_speedup_best"] = round(t1 / best, 3)
         res["rows"].append(row)
         del forests
+        for hh in hs[1:]:
+            hh.close()
         torch.cuda.empty_cache()
     print(json.dumps(res))
 
