@@ -35,9 +35,10 @@ def main():
     d = sys.argv[1]
     data = defaultdict(dict)
     for p in glob.glob(os.path.join(d, "l2rw_*_J*.csv")):
-        m = re.search(r"l2rw_(C\d)_J(\d)\.csv$", p)
+        m = re.search(r"l2rw_(C\d)_J(\d|p)\.csv$", p)
         if m:
-            data[m.group(1)][int(m.group(2))] = load(p)
+            j = m.group(2)
+            data[m.group(1)][0 if j == "p" else int(j)] = load(p)
     out = {}
     for c in sorted(data):
         j4 = data[c].get(4)
@@ -52,6 +53,13 @@ def main():
             if j in data[c]:
                 row[f"Jump{j}_read_rel"] = round(rd(data[c][j]) / rd(j4), 3)
                 row[f"Jump{j}_write_rel"] = round(wr(data[c][j]) / max(wr(j4), 1), 3)
+        jp = data[c].get(0)      # Jump4 on the plain path (batch 0): Jump1-3's own path
+        if jp:
+            row["jump4_plain_read_per_write"] = round(rd(jp) / max(wr(jp), 1), 2)
+            for j in (1, 2, 3):
+                if j in data[c]:
+                    row[f"Jump{j}_read_rel_plain"] = round(rd(data[c][j]) / rd(jp), 3)
+                    row[f"Jump{j}_write_rel_plain"] = round(wr(data[c][j]) / max(wr(jp), 1), 3)
         out[c] = row
     print(json.dumps(out, indent=1))
 
