@@ -309,7 +309,12 @@ typedef enum {
                                      R21 bitmap (anchor-tree membership proofs) to skip
                                      walks; merge_encoded extends the bitmap with the
                                      vertices it joins to the anchor's tree.  0 (default)
-                                     = no such assumption.                             */
+                                     = no such assumption.                             */,
+    ECL_CC_OPT_VEC = 21           /* 1 = hook_warp / hook_block stream the adjacency as
+                                     aligned 16-byte quads (R31; used when
+                                     nlist is 16-byte aligned, else scalar loads),
+                                     0 (default; measured faster at C5) = four-byte
+                                     loads.  Labels unchanged.                         */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 

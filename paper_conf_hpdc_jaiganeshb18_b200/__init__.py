@@ -48,6 +48,7 @@ OPT = {
     "flatten_passes": 18,
     "fuse_init": 19,
     "merge_filter": 20,
+    "vec": 21,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 

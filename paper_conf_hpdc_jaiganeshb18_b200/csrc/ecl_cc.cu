@@ -119,6 +119,8 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.gbits = nullptr;
     p.fa = h->fa;
     p.fb = h->fb;
+    // R31: quads need a 16-byte aligned adjacency base (quad q = entries 4q..4q+3)
+    p.vec = h->vec && ((reinterpret_cast<uintptr_t>(nlist) & 15) == 0);
     {
         // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
         const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
@@ -183,13 +185,19 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, tiles * kWarp, sm, h->occ_thread), kBlock, sm, s>>>(p);
         };
+        // R31 quad engine as its own instantiation (the scalar kernels keep their
+        // register allocation)
+        void (*const front_k)(Params) = p.vec ? hook_range_kernel<MODE, idx_t, kUnitFront, true, true>
+                                              : hook_range_kernel<MODE, idx_t, kUnitFront, true, false>;
+        void (*const back_k)(Params) = p.vec ? hook_range_kernel<MODE, idx_t, kUnitBack, false, true>
+                                             : hook_range_kernel<MODE, idx_t, kUnitBack, false, false>;
         auto warp_k = [&] {
-            auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
+            auto k = front_k;
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
         };
         auto block_k = [&] {
-            auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
+            auto k = back_k;
             const size_t sm = hook_smem_bytes<idx_t>();
             k<<<grid_for(h, (const void *)k, -1, sm, h->occ_range), kBlock, sm, s>>>(p);
         };
@@ -197,8 +205,7 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             // concurrent: hub chunks (L2-request bound) on a side stream next to the
             // warp and thread bins (issue / latency bound), occupancy split per SM
             const size_t sm = hook_smem_bytes<idx_t>();
-            const int full = blocks_per_sm(
-                h, (const void *)hook_range_kernel<MODE, idx_t, kUnitFront, true>, sm);
+            const int full = blocks_per_sm(h, (const void *)front_k, sm);
             // hook_block is launched first with a capped grid; hook_warp / hook_thread get
             // full persistent grids whose surplus blocks start as hook_block's retire (a
             // graph without hubs gives the whole GPU to the other two at once)
@@ -213,18 +220,19 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             CK(cudaStreamWaitEvent(h->side, h->fork, 0), "fork wait");
             if (tm) cudaEventRecord(h->ev[6], h->side);
             {
-                auto k = hook_range_kernel<MODE, idx_t, kUnitBack, false>;
+                auto k = back_k;
                 k<<<grid_for(h, (const void *)k, -1, sm, cb), kBlock, sm, h->side>>>(p);
             }
             if (tm) cudaEventRecord(h->ev[7], h->side);
             {
                 auto k = hook_thread_kernel<MODE, idx_t>;
                 const long long tiles = (nrows + kWarp - 1) / kWarp;
-                k<<<grid_for(h, (const void *)k, tiles * kWarp, sm, cw), kBlock, sm, s>>>(p);
+                const size_t smt = hook_smem_bytes<idx_t>();
+                k<<<grid_for(h, (const void *)k, tiles * kWarp, smt, cw), kBlock, smt, s>>>(p);
             }
             mark(2);
             {
-                auto k = hook_range_kernel<MODE, idx_t, kUnitFront, true>;
+                auto k = front_k;
                 k<<<grid_for(h, (const void *)k, -1, sm, cw), kBlock, sm, s>>>(p);
             }
             mark(3);
@@ -800,6 +808,9 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         break;
     case ECL_CC_OPT_MERGE_FILTER:
         h->merge_filter = value != 0;
+        break;
+    case ECL_CC_OPT_VEC:
+        h->vec = value != 0;
         break;
     case ECL_CC_OPT_FUSE_INIT:
         if (value < 0 || value > 2) return fail_arg(h, "fuse_init must be 0, 1 or 2");

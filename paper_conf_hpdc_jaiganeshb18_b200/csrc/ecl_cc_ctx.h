@@ -53,9 +53,10 @@ struct ecl_cc_ctx {
     unsigned *gbits = nullptr;            // R21 bitmap (grow-only)
     size_t gbits_words = 0;
     bool gbits_live = false;              // the last run used the R21 bitmap
-    int last_lazy = 0;
+    int last_lazy = 0;                    // the last run's R28 mode (0 off, 1 on, 2 probe)
     int merge_filter = 0;                 // merge_encoded / finalize use the last run's R21
-                                          //   bitmap as membership proofs (multi-GPU)                    // the last run's R28 mode (0 off, 1 on, 2 probe)
+                                          //   bitmap as membership proofs (multi-GPU)
+    int vec = 0;                          // R31 quad engine in hook_warp / hook_block
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks
