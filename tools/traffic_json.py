@@ -2,6 +2,7 @@
 from ncu --metrics logs written by tools/gpu_profile.sh.
 
     python tools/traffic_json.py TAG   # reads gpurun_out/TAG_traffic_C{1..5}.csv
+    python tools/traffic_json.py DIR   # reads DIR/traffic_C{1..5}.csv (tools/gpu_final.sh)
 """
 import json
 import os
@@ -17,6 +18,8 @@ def main(tag):
     out = {}
     for c in ("C1", "C2", "C3", "C4", "C5"):
         path = os.path.join(ROOT, "gpurun_out", f"{tag}_traffic_{c}.csv")
+        if os.path.isdir(tag):                  # tools/gpu_final.sh layout: DIR/traffic_Cn.csv
+            path = os.path.join(tag, f"traffic_{c}.csv")
         if not os.path.exists(path):
             continue
         per = load(path)
