@@ -29,3 +29,35 @@ def test_full_size_exact(name):
     bad = np.nonzero(got != expect)[0]
     assert bad.size == 0, f"{name}: {bad.size} labels differ (first v={bad[0]})"
     assert oracle.check(nidx, nl, got, ncc) == 0
+
+
+_EXPECT = {}
+
+
+def _expect(name, g):
+    if name not in _EXPECT:
+        nidx, nl = g.numpy()
+        _EXPECT[name] = oracle.bfs(nidx, nl)
+    return _EXPECT[name]
+
+
+@pytest.mark.parametrize("name", ["C3", "C4", "C5"])
+def test_full_size_option_variants(name):
+    """The same full-size graphs under the non-default memory model and kernel paths:
+    load_mode 0 (every racing parent[] load ld.relaxed.gpu, SURVEY R7 as written;
+    DESIGN.md §5 "Memory model"), the paper's sequential kernel order 0, and the
+    R31 16-byte quad engine."""
+    g = gg.make_config(name, seed=1, device="cuda")
+    expect, ncc = _expect(name, g)
+    variants = [{"load_mode": 0}, {"order": 0}, {"vec": 1}, {"load_mode": 0, "order": 0}]
+    with ecl.Handle(0) as h:
+        for opts in variants:
+            for k, v in opts.items():
+                h.set_option(k, v)
+            got = h.run(g.nindex, g.nlist).cpu().numpy()
+            for k in opts:
+                h.set_option(k, {"load_mode": 1, "order": 2, "vec": 0}[k])
+            bad = np.nonzero(got != expect)[0]
+            assert bad.size == 0, f"{name} {opts}: {bad.size} labels differ (first v={bad[0]})"
+    nidx, nl = g.numpy()
+    assert oracle.check(nidx, nl, got, ncc) == 0

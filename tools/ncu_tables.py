@@ -19,6 +19,10 @@ def kname(s):
         return "hook_warp" if re.search(r"16,\s*(1|true)", s) else "hook_block"
     if "finalize" in s:
         return "finalize"
+    if "locality_probe" in s:
+        return "locality_probe"
+    if "fused_small" in s:
+        return "fused"
     if "prejump" in s:
         return "prejump"
     if "depth_probe" in s:

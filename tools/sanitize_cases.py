@@ -43,7 +43,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--variants", action="store_true",
-                    help="also the ablation paths (Jump1-3, batch 0, Init1/2, Fini1/2)")
+                    help="also the ablation paths (Jump1-3, batch 0, Init1/2, Fini1/2) and "
+                         "the R31 quad engine")
     args = ap.parse_args()
     bad = 0
     runs = 0
@@ -66,7 +67,8 @@ def main():
                                 bad += 1
             if args.variants:
                 for opts in (dict(jump=1), dict(jump=2), dict(jump=3), dict(batch=0),
-                             dict(init=1, fini=1), dict(init=2, fini=2)):
+                             dict(init=1, fini=1), dict(init=2, fini=2), dict(vec=1),
+                             dict(vec=1, thresh_thread=2, thresh_warp=20, filter=1)):
                     for k, v in opts.items():
                         h.set_option(k, v)
                     out = h.run(gd.nindex, gd.nlist)
@@ -76,7 +78,9 @@ def main():
                         print(f"MISMATCH {g.name} {opts}", flush=True)
                         bad += 1
                     for k in opts:
-                        h.set_option(k, {"jump": 4, "batch": 1, "init": 3, "fini": 3}[k])
+                        h.set_option(k, {"jump": 4, "batch": 1, "init": 3, "fini": 3, "vec": 0,
+                                         "thresh_thread": 16, "thresh_warp": 352,
+                                         "filter": filt}[k])
             h.set_option("order", 2).set_option("prejump", 1).set_option("filter", 2)
             lab, ta, tb = h.spanning_forest(gd.nindex, gd.nlist)
             torch.cuda.synchronize()
