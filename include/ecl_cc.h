@@ -314,7 +314,16 @@ typedef enum {
                                      aligned 16-byte quads (R31; used when
                                      nlist is 16-byte aligned, else scalar loads),
                                      0 (default; measured faster at C5) = four-byte
-                                     loads.  Labels unchanged.                         */
+                                     loads.  Labels unchanged.                         */,
+    ECL_CC_OPT_FUSED = 22         /* R33: the whole path as ONE cooperative
+                                     launch (grid barriers between init, the R23
+                                     passes, the three hook kernels and finalize):
+                                     0 off, 1 on, 2 (default) for graphs with at most
+                                     2^18 rows and 2^22 entries.  Not used by
+                                     ecl_cc_run_rows or with ECL_CC_OPT_TIMING (no
+                                     per-phase events inside one kernel); the kernel
+                                     ORDER option does not apply to it.  Labels
+                                     unchanged.                                        */
 } ecl_cc_option;
 ECL_CC_API ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value);
 
@@ -344,7 +353,8 @@ ECL_CC_API ecl_cc_status ecl_cc_get_stats_ex(ecl_cc_handle h, int64_t *out, int 
 /* Debug: what the most recent run decided (synchronises it); count <= 4:
  * [0] 1 if Init3 ran inside the hook kernels (R28), [1] 1 if the R23 depth probe found a
  * deep forest (the pointer-jumping passes ran), [2] 1 if the R21 bitmap filter was on,
- * [3] the R21 anchor vertex (-1 if none). */
+ * [3] the R21 anchor vertex (-1 if none), [4] 1 if the run took the R33 single-launch
+ * path.  count <= 5. */
 ECL_CC_API ecl_cc_status ecl_cc_get_run_info(ecl_cc_handle h, int64_t *out, int count);
 
 /* Debug: the handle's R21 anchor-tree membership bitmap (R21) as left by the

@@ -49,6 +49,7 @@ OPT = {
     "fuse_init": 19,
     "merge_filter": 20,
     "vec": 21,
+    "fused": 22,
 }
 PHASES = ("init_bin", "hook_thread", "hook_warp", "hook_block", "finalize")
 
@@ -397,10 +398,10 @@ class Handle:
 
     def run_info(self) -> dict:
         """Decisions of the last run (ecl_cc_get_run_info)."""
-        arr = (ctypes.c_int64 * 4)()
-        self._check(self._lib.ecl_cc_get_run_info(self._h, arr, 4))
+        arr = (ctypes.c_int64 * 5)()
+        self._check(self._lib.ecl_cc_get_run_info(self._h, arr, 5))
         return {"lazy_init3": bool(arr[0]), "deep_forest_passes": bool(arr[1]),
-                "filter": bool(arr[2]), "anchor": int(arr[3])}
+                "filter": bool(arr[2]), "anchor": int(arr[3]), "fused": bool(arr[4])}
 
     def filter_bitmap(self):
         """(device address or None, words, anchor) of the R21 bitmap of the last run."""

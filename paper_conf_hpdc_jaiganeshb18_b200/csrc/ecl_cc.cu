@@ -26,6 +26,9 @@ constexpr int kNumStats = 16;
 #define ECL_FAST_FINI 1
 #endif
 constexpr bool kFastFini = ECL_FAST_FINI != 0;   // Fini3 via finalize3_kernel
+// R33 auto mode: the single-launch path for graphs up to this size
+constexpr int kFusedMaxRows = 1 << 18;
+constexpr long long kFusedMaxEntries = 1LL << 22;
 
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
 
@@ -137,6 +140,30 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
             CK(cudaMemsetAsync(h->gbits, 0, words * 4, s), "cudaMemsetAsync(gbits)");
             p.gbits = h->gbits;
         }
+    }
+
+    // R33: the whole path as one cooperative launch for small graphs (no per-phase
+    // timing events inside it, so ECL_CC_OPT_TIMING keeps the multi-kernel path)
+    const bool fuse = !rows_mode && h->timing == 0 && h->stop_after != 1 && nrows > 0 &&
+                      (h->fused == 1 ||
+                       (h->fused == 2 && nrows <= kFusedMaxRows && m <= kFusedMaxEntries));
+    h->last_fused = fuse;
+    if (fuse) {
+        auto k = fused_small_kernel<MODE, idx_t>;
+        const size_t sm = fused_smem_bytes<idx_t>();
+        const int cap = h->sms * blocks_per_sm(h, (const void *)k, sm);
+        long long want = std::max<long long>(h->sms, ((long long)nrows + kBlock - 1) / kBlock);
+        if (h->grid_blocks > 0) want = h->grid_blocks;
+        const int blocks = (int)std::min<long long>(cap, want);
+        FusedArgs fa;
+        fa.prejump = h->prejump;
+        fa.fini = h->stop_after == 2 ? 0 : h->fini;
+        fa.ctl = (int *)(h->cnt + 4);
+        fa.bar = (unsigned *)(h->cnt + 12);
+        void *args[] = {&p, &fa};
+        CK(cudaLaunchCooperativeKernel((const void *)k, dim3(blocks), dim3(kBlock), args, sm, s),
+           "fused launch");
+        return ECL_CC_OK;
     }
 
     const bool tm = h->timing != 0;
@@ -809,6 +836,10 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
     case ECL_CC_OPT_MERGE_FILTER:
         h->merge_filter = value != 0;
         break;
+    case ECL_CC_OPT_FUSED:
+        if (value < 0 || value > 2) return fail_arg(h, "fused must be 0, 1 or 2");
+        h->fused = (int)value;
+        break;
     case ECL_CC_OPT_VEC:
         h->vec = value != 0;
         break;
@@ -863,16 +894,16 @@ ecl_cc_status ecl_cc_get_worklist(ecl_cc_handle h, int32_t *front, int64_t *nfro
 
 ecl_cc_status ecl_cc_get_run_info(ecl_cc_handle h, int64_t *out, int count)
 {
-    if (!h || !out || count < 0 || count > 4) return ECL_CC_ERR_INVALID_ARG;
+    if (!h || !out || count < 0 || count > 5) return ECL_CC_ERR_INVALID_ARG;
     DeviceGuard g(h->device);
     unsigned long long c[11] = {};
     CK(cudaStreamSynchronize(h->last_stream), "sync");
     CK(cudaMemcpy(c, h->cnt, sizeof(c), cudaMemcpyDeviceToHost), "D2H counters");
     const int *ctl = (const int *)(c + 4);
     const int lazy_flag = (int)(unsigned)c[7];
-    const int64_t v[4] = {h->last_lazy == 1 || (h->last_lazy == 2 && lazy_flag) ? 1 : 0,
+    const int64_t v[5] = {h->last_lazy == 1 || (h->last_lazy == 2 && lazy_flag) ? 1 : 0,
                           ctl[0] ? 1 : 0, h->gbits_live ? 1 : 0,
-                          c[10] ? (int64_t)(unsigned)c[10] : -1};
+                          c[10] ? (int64_t)(unsigned)c[10] : -1, h->last_fused ? 1 : 0};
     for (int i = 0; i < count; i++) out[i] = v[i];
     return ECL_CC_OK;
 }

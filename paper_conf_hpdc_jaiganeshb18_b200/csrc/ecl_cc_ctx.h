@@ -57,6 +57,8 @@ struct ecl_cc_ctx {
     int merge_filter = 0;                 // merge_encoded / finalize use the last run's R21
                                           //   bitmap as membership proofs (multi-GPU)
     int vec = 0;                          // R31 quad engine in hook_warp / hook_block
+    int fused = 2;                        // R33 single launch: 0 off, 1 on, 2 small graphs
+    bool last_fused = false;              // the last run took the single-launch path
     int stop_after = 0;
     int load_mode = 1;
     int ttas = 1;                         // test-and-test-and-set hooks

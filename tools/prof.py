@@ -39,10 +39,13 @@ def main():
     ap.add_argument("--prejump", type=int, default=2)
     ap.add_argument("--fuse", type=int, default=2, help="ECL_CC_OPT_FUSE_INIT (R28)")
     ap.add_argument("--vec", type=int, default=0, help="ECL_CC_OPT_VEC (R31 quad engine)")
+    ap.add_argument("--fused", type=int, default=2, help="ECL_CC_OPT_FUSED (R33 single launch)")
+    ap.add_argument("--timing", type=int, default=1,
+                    help="per-phase events (1; the multi-kernel path) or 0 (run span only)")
     args = ap.parse_args()
     g = gg.make_config(args.config, seed=args.seed, device="cuda", scale_down=args.scale_down)
     h = ecl.Handle(0, stats=args.stats)
-    h.set_option("load_mode", args.mode).set_option("timing", 1)
+    h.set_option("load_mode", args.mode).set_option("timing", args.timing)
     h.set_option("thresh_thread", args.t1).set_option("thresh_warp", args.t2)
     h.set_option("grid_blocks", args.grid).set_option("ttas", args.ttas)
     h.set_option("l2_fetch", args.l2fetch)
@@ -53,6 +56,8 @@ def main():
     h.set_option("order", args.order).set_option("prejump", args.prejump)
     if args.vec:
         h.set_option("vec", args.vec)
+    if args.fused != 2:
+        h.set_option("fused", args.fused)
     if args.fuse != 2:
         h.set_option("fuse_init", args.fuse)
     out = torch.empty(g.n, dtype=torch.int32, device="cuda")
@@ -62,13 +67,13 @@ def main():
         e0.record()
         h.run(g.nindex, g.nlist, out=out)
         e1.record()
-        t = h.timing()
+        t = h.timing() if args.timing else {}
         # the run's own span: with order 2 the hook kernels overlap (phases sum to more)
         e1.synchronize()
         t["total"] = e0.elapsed_time(e1)
         res.append(t)
     best = min(res, key=lambda r: r["total"])
-    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "order": args.order, "prejump": args.prejump, "fuse": args.fuse, "vec": args.vec, "n": g.n, "m": g.m, "mode": args.mode,
+    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "order": args.order, "prejump": args.prejump, "fuse": args.fuse, "vec": args.vec, "fused": h.run_info()["fused"], "n": g.n, "m": g.m, "mode": args.mode,
             "best_ms": {k: round(v, 4) for k, v in best.items()},
             "medges_s": round(g.m / best["total"] / 1e3, 1)}
     if args.stats:
