@@ -313,13 +313,15 @@ typedef enum {
     ECL_CC_OPT_VEC = 21           /* 1 = hook_warp / hook_block stream the adjacency as
                                      aligned 16-byte quads (R31; used when
                                      nlist is 16-byte aligned, else scalar loads),
-                                     0 (default; measured faster at C5) = four-byte
-                                     loads.  Labels unchanged.                         */,
+                                     0 = four-byte loads, 2 (default) = quads with
+                                     int32 offsets (ecl_cc_run), four-byte loads with
+                                     int64 offsets (measured: C4 faster with quads, C5
+                                     slower).  Labels unchanged.                       */,
     ECL_CC_OPT_FUSED = 22         /* R33: the whole path as ONE cooperative
                                      launch (grid barriers between init, the R23
                                      passes, the three hook kernels and finalize):
                                      0 off, 1 on, 2 (default) for graphs with at most
-                                     2^18 rows and 2^22 entries.  Not used by
+                                     2^20 rows and 2^22 entries.  Not used by
                                      ecl_cc_run_rows or with ECL_CC_OPT_TIMING (no
                                      per-phase events inside one kernel); the kernel
                                      ORDER option does not apply to it.  Labels

@@ -26,8 +26,10 @@ constexpr int kNumStats = 16;
 #define ECL_FAST_FINI 1
 #endif
 constexpr bool kFastFini = ECL_FAST_FINI != 0;   // Fini3 via finalize3_kernel
-// R33 auto mode: the single-launch path for graphs up to this size
-constexpr int kFusedMaxRows = 1 << 18;
+// R33 auto mode: the single-launch path for graphs up to this size (measured crossover,
+// profiles/r2/ab_fused_size_r2z: faster up to ~4 M entries on every family; at ~8 M
+// entries slower on R-MAT, whose hub chunks want more blocks than one per SM)
+constexpr int kFusedMaxRows = 1 << 20;
 constexpr long long kFusedMaxEntries = 1LL << 22;
 
 const char *kVersion = "ecl_cc-b200 0.1 (sm_100a)";
@@ -122,8 +124,11 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.gbits = nullptr;
     p.fa = h->fa;
     p.fb = h->fb;
-    // R31: quads need a 16-byte aligned adjacency base (quad q = entries 4q..4q+3)
-    p.vec = h->vec && ((reinterpret_cast<uintptr_t>(nlist) & 15) == 0);
+    // R31: quads need a 16-byte aligned adjacency base (quad q = entries 4q..4q+3); auto
+    // (2): on with int32 offsets only — with int64 offsets the quad kernels' extra 64-bit
+    // state spills at the 32-register cap (C4: -6 %, C5: +4 %, profiles/r2/ab_quads_*)
+    p.vec = (h->vec == 1 || (h->vec == 2 && sizeof(idx_t) == 4)) &&
+            ((reinterpret_cast<uintptr_t>(nlist) & 15) == 0);
     {
         // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
         const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
@@ -152,7 +157,9 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         auto k = fused_small_kernel<MODE, idx_t>;
         const size_t sm = fused_smem_bytes<idx_t>();
         const int cap = h->sms * blocks_per_sm(h, (const void *)k, sm);
-        long long want = std::max<long long>(h->sms, ((long long)nrows + kBlock - 1) / kBlock);
+        // one block per SM: on C1 148 blocks ran 0.082 ms, 256 / 296 / 592 blocks
+        // 0.09 / 0.09-0.10 / 0.115 ms (fewer CAS collisions, cheaper grid barriers)
+        long long want = h->sms;
         if (h->grid_blocks > 0) want = h->grid_blocks;
         const int blocks = (int)std::min<long long>(cap, want);
         FusedArgs fa;
@@ -841,7 +848,8 @@ ecl_cc_status ecl_cc_set_option(ecl_cc_handle h, int option, int64_t value)
         h->fused = (int)value;
         break;
     case ECL_CC_OPT_VEC:
-        h->vec = value != 0;
+        if (value < 0 || value > 2) return fail_arg(h, "vec must be 0, 1 or 2");
+        h->vec = (int)value;
         break;
     case ECL_CC_OPT_FUSE_INIT:
         if (value < 0 || value > 2) return fail_arg(h, "fuse_init must be 0, 1 or 2");

@@ -49,14 +49,15 @@ def test_full_size_option_variants(name):
     R31 16-byte quad engine."""
     g = gg.make_config(name, seed=1, device="cuda")
     expect, ncc = _expect(name, g)
-    variants = [{"load_mode": 0}, {"order": 0}, {"vec": 1}, {"load_mode": 0, "order": 0}]
+    variants = [{"load_mode": 0}, {"order": 0}, {"vec": 1}, {"vec": 0},
+                {"load_mode": 0, "order": 0}]
     with ecl.Handle(0) as h:
         for opts in variants:
             for k, v in opts.items():
                 h.set_option(k, v)
             got = h.run(g.nindex, g.nlist).cpu().numpy()
             for k in opts:
-                h.set_option(k, {"load_mode": 1, "order": 2, "vec": 0}[k])
+                h.set_option(k, {"load_mode": 1, "order": 2, "vec": 2}[k])
             bad = np.nonzero(got != expect)[0]
             assert bad.size == 0, f"{name} {opts}: {bad.size} labels differ (first v={bad[0]})"
     nidx, nl = g.numpy()

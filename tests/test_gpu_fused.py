@@ -118,7 +118,7 @@ def test_fused_spanning_forest(h):
 def test_fused_auto_choice(h):
     small = gg.make_config("C1", seed=1)
     assert check(h, small) is True                      # auto: C1 takes the single launch
-    big = gg.make_config("C4", seed=1, scale_down=4)    # 2^20 rows: above the threshold
+    big = gg.make_config("C4", seed=1, scale_down=4)    # 2^20 rows, 2^25 entries: above
     assert check(h, big) is False
     assert check(h, small, fused=0) is False
 

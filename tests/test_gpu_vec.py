@@ -31,7 +31,7 @@ def run_opts(h, nindex, nlist, **opts):
         out = h.run(nindex, nlist)
         torch.cuda.synchronize()
     finally:
-        h.set_option("vec", 0).set_option("order", 2).set_option("filter", 2)
+        h.set_option("vec", 2).set_option("order", 2).set_option("filter", 2)
         h.set_option("thresh_thread", 16).set_option("thresh_warp", 352)
     return out.cpu().numpy()
 
@@ -51,7 +51,7 @@ def misaligned(nlist, shift):
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-@pytest.mark.parametrize("vec", [0, 1])
+@pytest.mark.parametrize("vec", [0, 1, 2])
 @pytest.mark.parametrize("order", [0, 2])
 def test_vec_configs(h, name, vec, order):
     g = gg.make_config(name, seed=3, scale_down=SMALL[name], device="cuda")

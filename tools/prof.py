@@ -38,7 +38,8 @@ def main():
     ap.add_argument("--order", type=int, default=2)
     ap.add_argument("--prejump", type=int, default=2)
     ap.add_argument("--fuse", type=int, default=2, help="ECL_CC_OPT_FUSE_INIT (R28)")
-    ap.add_argument("--vec", type=int, default=0, help="ECL_CC_OPT_VEC (R31 quad engine)")
+    ap.add_argument("--vec", type=int, default=-1,
+                    help="ECL_CC_OPT_VEC (R31 quad engine; -1 = library default)")
     ap.add_argument("--fused", type=int, default=2, help="ECL_CC_OPT_FUSED (R33 single launch)")
     ap.add_argument("--timing", type=int, default=1,
                     help="per-phase events (1; the multi-kernel path) or 0 (run span only)")
@@ -54,7 +55,7 @@ def main():
     h.set_option("filter", args.filter)
     h.set_option("init", args.init).set_option("fini", args.fini)
     h.set_option("order", args.order).set_option("prejump", args.prejump)
-    if args.vec:
+    if args.vec >= 0:
         h.set_option("vec", args.vec)
     if args.fused != 2:
         h.set_option("fused", args.fused)
@@ -73,7 +74,7 @@ def main():
         t["total"] = e0.elapsed_time(e1)
         res.append(t)
     best = min(res, key=lambda r: r["total"])
-    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "order": args.order, "prejump": args.prejump, "fuse": args.fuse, "vec": args.vec, "fused": h.run_info()["fused"], "n": g.n, "m": g.m, "mode": args.mode,
+    line = {"config": args.config, "lib": os.path.basename(ecl.library_path()), "ttas": args.ttas, "occ": [args.occ_thread, args.occ_range], "bjif": [args.batch, args.jump, args.init, args.fini], "filter": args.filter, "order": args.order, "prejump": args.prejump, "fuse": args.fuse, "vec": args.vec, "grid": args.grid, "fused": h.run_info()["fused"], "n": g.n, "m": g.m, "mode": args.mode,
             "best_ms": {k: round(v, 4) for k, v in best.items()},
             "medges_s": round(g.m / best["total"] / 1e3, 1)}
     if args.stats:

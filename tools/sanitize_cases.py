@@ -78,7 +78,7 @@ def main():
                         print(f"MISMATCH {g.name} {opts}", flush=True)
                         bad += 1
                     for k in opts:
-                        h.set_option(k, {"jump": 4, "batch": 1, "init": 3, "fini": 3, "vec": 0,
+                        h.set_option(k, {"jump": 4, "batch": 1, "init": 3, "fini": 3, "vec": 2,
                                          "thresh_thread": 16, "thresh_warp": 352,
                                          "filter": filt}[k])
             h.set_option("order", 2).set_option("prejump", 1).set_option("filter", 2)
