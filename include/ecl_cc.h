@@ -310,13 +310,14 @@ typedef enum {
                                      walks; merge_encoded extends the bitmap with the
                                      vertices it joins to the anchor's tree.  0 (default)
                                      = no such assumption.                             */,
-    ECL_CC_OPT_VEC = 21           /* 1 = hook_warp / hook_block stream the adjacency as
-                                     aligned 16-byte quads (R31; used when
-                                     nlist is 16-byte aligned, else scalar loads),
-                                     0 = four-byte loads, 2 (default) = quads with
-                                     int32 offsets (ecl_cc_run), four-byte loads with
-                                     int64 offsets (measured: C4 faster with quads, C5
-                                     slower).  Labels unchanged.                       */,
+    ECL_CC_OPT_VEC = 21           /* 1 = hook_warp and hook_block stream the adjacency
+                                     as aligned 16-byte quads (R31; used when
+                                     nlist is 16-byte aligned and m < 2^33, else
+                                     four-byte loads), 2 (default) = hook_warp only and
+                                     only with int32 offsets (quads help its multi-row
+                                     rounds, not the hubs' single-row rounds; measured
+                                     slower with int64 offsets), 0 = four-byte loads
+                                     everywhere.  Labels unchanged.                    */,
     ECL_CC_OPT_FUSED = 22         /* R33: the whole path as ONE cooperative
                                      launch (grid barriers between init, the R23
                                      passes, the three hook kernels and finalize):

@@ -124,11 +124,13 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
     p.gbits = nullptr;
     p.fa = h->fa;
     p.fb = h->fb;
-    // R31: quads need a 16-byte aligned adjacency base (quad q = entries 4q..4q+3); auto
-    // (2): on with int32 offsets only — with int64 offsets the quad kernels' extra 64-bit
-    // state spills at the 32-register cap (C4: -6 %, C5: +4 %, profiles/r2/ab_quads_*)
-    p.vec = (h->vec == 1 || (h->vec == 2 && sizeof(idx_t) == 4)) &&
-            ((reinterpret_cast<uintptr_t>(nlist) & 15) == 0);
+    // R31: quads need a 16-byte aligned adjacency base (quad q = entries 4q..4q+3) and
+    // 32-bit quad indices (m < 2^33).  p.vec: bit 0 hook_warp, bit 1 hook_block.  Default
+    // (2): hook_warp only, and only with int32 offsets — quads cut the multi-piece
+    // rounds' per-entry owner work (C4: 2.23 vs 2.33 ms) but cost the hubs' uniform rounds
+    // (hook_block) and, with int64 offsets, hook_warp too (C5 hook_warp 3.75 vs 3.56 ms)
+    const bool quads_ok = ((reinterpret_cast<uintptr_t>(nlist) & 15) == 0) && m < (1LL << 33);
+    p.vec = !quads_ok ? 0 : h->vec == 1 ? 3 : (h->vec == 2 && sizeof(idx_t) == 4) ? 1 : 0;
     {
         // auto: on when parent[] (4n bytes) cannot stay in the 126 MB L2
         const bool on = h->filter == 1 || (h->filter == 2 && (long long)n * 4 > (128ll << 20));
@@ -221,9 +223,9 @@ ecl_cc_status launch_path(ecl_cc_handle h, int n, long long m, int row_lo, int n
         };
         // R31 quad engine as its own instantiation (the scalar kernels keep their
         // register allocation)
-        void (*const front_k)(Params) = p.vec ? hook_range_kernel<MODE, idx_t, kUnitFront, true, true>
+        void (*const front_k)(Params) = (p.vec & 1) ? hook_range_kernel<MODE, idx_t, kUnitFront, true, true>
                                               : hook_range_kernel<MODE, idx_t, kUnitFront, true, false>;
-        void (*const back_k)(Params) = p.vec ? hook_range_kernel<MODE, idx_t, kUnitBack, false, true>
+        void (*const back_k)(Params) = (p.vec & 2) ? hook_range_kernel<MODE, idx_t, kUnitBack, false, true>
                                              : hook_range_kernel<MODE, idx_t, kUnitBack, false, false>;
         auto warp_k = [&] {
             auto k = front_k;

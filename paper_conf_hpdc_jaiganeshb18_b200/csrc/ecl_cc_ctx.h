@@ -56,7 +56,8 @@ struct ecl_cc_ctx {
     int last_lazy = 0;                    // the last run's R28 mode (0 off, 1 on, 2 probe)
     int merge_filter = 0;                 // merge_encoded / finalize use the last run's R21
                                           //   bitmap as membership proofs (multi-GPU)
-    int vec = 2;                          // R31 quad engine: 0 off, 1 on, 2 int32 offsets
+    int vec = 2;                          // R31 quad engine: 0 off, 1 both range kernels,
+                                          //   2 hook_warp with int32 offsets
     int fused = 2;                        // R33 single launch: 0 off, 1 on, 2 small graphs
     bool last_fused = false;              // the last run took the single-launch path
     int stop_after = 0;
