@@ -367,6 +367,15 @@ def launches_per_step(world: int, rank: int, chunks: int, merge: str, probe: int
     return 7 + recv * chunks + (1 if rank == 0 else 0)
 
 
+def launches_per_run(info: dict, world: int, rank: int, chunks: int, merge: str,
+                     probe: int = 0) -> int:
+    """Our kernels per timed step: ONE when the run took the R33 single-launch path
+    (info["single_launch"], from ecl_cc_get_run_info), else launches_per_step."""
+    if world == 1 and info.get("single_launch"):
+        return 1
+    return launches_per_step(world, rank, chunks, merge, probe)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -668,9 +677,8 @@ def main():
                        "partition": "row_weights" + (" + calibrated" if calib else ""),
                        "calibration_forest_ms": calib}
                       if world > 1 else {})},
-        "gpu_launches": (1 if info.get("single_launch") else
-                         launches_per_step(world, rank, args.chunks, args.merge,
-                                           probe=int(m < 16 * n))) * args.steps,
+        "gpu_launches": launches_per_run(info, world, rank, args.chunks, args.merge,
+                                         probe=int(m < 16 * n)) * args.steps,
         "clocks": clk.summary(),
         "roofline": roof,
         "phase_ms": {k: round(v, 4) for k, v in phase.items()},

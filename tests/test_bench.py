@@ -111,3 +111,14 @@ def test_gpus_flag_must_match_world():
                         "--steps", "1", "--config", "C1"], capture_output=True, text=True,
                        env=env, timeout=300)
     assert r.returncode != 0 and "WORLD_SIZE=3" in r.stderr
+
+
+def test_single_launch_counts_one_kernel_per_step():
+    # R33: a run that took the single-launch path is ONE kernel (fused_small_kernel);
+    # the multi-kernel count applies otherwise
+    import bench
+    assert bench.launches_per_run({"single_launch": True}, 1, 0, 4, "p2p", probe=1) == 1
+    assert bench.launches_per_run({"single_launch": False}, 1, 0, 4, "p2p") == 7
+    assert bench.launches_per_run({}, 1, 0, 4, "p2p", probe=1) == 8
+    assert bench.launches_per_run({"single_launch": True}, 2, 0, 4, "p2p") == \
+        bench.launches_per_step(2, 0, 4, "p2p")

@@ -136,3 +136,14 @@ def test_fused_repeat_and_stream(h):
     expect, _ = oracle.bfs(*g.numpy())
     for o in outs:
         assert np.array_equal(o.cpu().numpy(), expect)
+
+
+def test_fused_and_vec_option_values(h):
+    # ECL_CC_OPT_FUSED / ECL_CC_OPT_VEC take 0, 1 or 2; anything else is INVALID_ARG
+    for name in ("fused", "vec"):
+        for bad in (-1, 3):
+            with pytest.raises(ecl.EclCCError):
+                h.set_option(name, bad)
+        for ok in (0, 1, 2):
+            h.set_option(name, ok)
+        h.set_option(name, 2)
